@@ -1,0 +1,180 @@
+/*
+ * include/cg.h — C ABI of the B200-native Core Graph hot path.
+ *
+ * Method: Jiang et al., "Core Graph: Exploiting Edge Centrality to Speedup
+ * the Evaluation of Iterative Graph Queries", EuroSys '24.  Citations
+ * "P:<line>" refer to lines of the paper text and the section /
+ * algorithm / table they sit in.  Readings of ambiguous passages (Q1..Q20)
+ * are listed in DESIGN.md.
+ *
+ * Conventions for every entry point:
+ *   - Returns cg_status; CG_OK == 0.  Nothing throws across the ABI.  On
+ *     error, cg_last_error() returns a thread-local detail string.
+ *   - "device" pointers are CUDA device memory on the graph's device,
+ *     "host" pointers are CPU memory (pinned memory is fastest).
+ *   - Input pointers are BORROWED: read during the call (or, for
+ *     stream-ordered calls, until the stream reaches the call) and never
+ *     retained.  Output buffers are caller-allocated.
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default
+ *     stream).  cg_query / cg_rmat_generate are stream-ordered and
+ *     asynchronous; cg_graph_create and cg_build synchronise `stream`.
+ *   - No PyTorch types appear here; the Python binding passes raw pointers
+ *     (torch tensors' data_ptr) and a raw stream handle.
+ *   - Internal device memory comes from the allocator installed with
+ *     cg_set_allocator (the Python binding installs PyTorch's caching
+ *     allocator), else cudaMalloc.
+ */
+#ifndef CG_H
+#define CG_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    CG_OK = 0,
+    CG_EINVAL = -1,        /* bad argument: null pointer, source >= n, n_src < 0, K <= 0 or K > n, bad enum */
+    CG_ENOMEM = -2,        /* device allocation failed */
+    CG_ECUDA = -3,         /* a CUDA runtime error (detail in cg_last_error) */
+    CG_ENOCG = -4,         /* cg_query(..., CG_MODE_2PHASE) before cg_build for that kind */
+    CG_EOVERFLOW = -5,     /* n >= 2^32-1, m >= 2^32, or (n-1)*w_max >= 2^32-1 (SSSP could wrap) */
+    CG_EUNSUPPORTED = -7,  /* feature not available on this device (e.g. no cooperative launch) */
+    CG_EINTERNAL = -8      /* internal invariant violated (e.g. iteration bound exceeded) */
+} cg_status;
+
+/* The six query kinds (north_star; Table 6 P:1496-1535 for SSSP/SSWP/SSNP/Viterbi/REACH;
+ * BFS = hop count, reading D1).  Value words are u32 for all kinds except
+ * VITERBI, whose value is an IEEE binary32 probability stored in the same 32-bit slot. */
+typedef enum { CG_SSSP = 0, CG_SSWP = 1, CG_SSNP = 2, CG_VITERBI = 3, CG_BFS = 4, CG_REACH = 5 } cg_kind;
+
+/* CG_MODE_2PHASE: Algorithm 3 — phase 1 on the Core Graph, phase 2 on G
+ * from the impacted set.  CG_MODE_FULL: the baseline, the same relaxation on G only. */
+typedef enum { CG_MODE_2PHASE = 0, CG_MODE_FULL = 1 } cg_mode;
+
+/* Hub set H of Algorithm 1: the K highest total-degree vertices (P:464-466,
+ * P:1669-1677, reading Q7), K uniformly sampled vertices with outdeg > 0 (north_star,
+ * reading D2), or caller-given ids. */
+typedef enum { CG_HUBS_TOPDEG = 0, CG_HUBS_SAMPLED = 1, CG_HUBS_GIVEN = 2 } cg_hub_policy;
+
+/* Which Core Graph construction: AUTO = Algorithm 1 (specialized) for
+ * SSSP/SSWP/SSNP/VITERBI and Algorithm 2 (general) for BFS/REACH
+ * (reading Q12). */
+typedef enum { CG_ALG_AUTO = 0, CG_ALG_SPECIALIZED = 1, CG_ALG_GENERAL = 2 } cg_cg_alg;
+
+typedef struct cg_graph_s* cg_graph; /* opaque: owns G (CSR), G^R (CSC) and the CGs on one device */
+
+/* Per-query counters (SURVEY §5 tracing; Table 5 / Fig 5 analogs).  Edge and update
+ * counts of the asynchronous GPU relaxation are NOT unique (they depend on timing);
+ * impacted / reached / precise_p1 ARE unique. */
+typedef struct {
+    int64_t iters_p1, iters_p2;      /* BSP iterations of phase 1 (CG) and phase 2 (G or FULL) */
+    int64_t edges_p1, edges_p2;      /* edges scanned by Process (Alg 3 l.24) */
+    int64_t updates_p1, updates_p2;  /* successful CASMIN/CASMAX EdgeFunction updates (l.26) */
+    int64_t frontier_p1, frontier_p2;/* sum over iterations of |Active| */
+    int64_t impacted;                /* |Active| at the start of phase 2 (Alg 3 l.15, reading Q4) */
+    int64_t reached;                 /* |{v != s : Val(v) != InitVal}| after the query */
+    int64_t precise_p1;              /* |{v != s reached : p1(v) == final(v)}| (Table 5, reading Q16);
+                                        -1 unless the query kept phase-1 values */
+} cg_stats;
+
+typedef void* (*cg_alloc_fn)(size_t bytes, void* stream, void* ctx);
+typedef void (*cg_free_fn)(void* ptr, void* stream, void* ctx);
+
+/* Install the device allocator used for all internal memory (NULL, NULL restores cudaMalloc). */
+cg_status cg_set_allocator(cg_alloc_fn alloc, cg_free_fn free_fn, void* ctx);
+
+/*
+ * Build G(V,E) on `device` from an edge list of m directed weighted edges
+ * (src[i] -> dst[i], weight w[i] >= 1), device pointers, borrowed.
+ * Canonicalises (reading Q14): drops self-loops, collapses parallel edges to the minimum
+ * weight, sorts rows by destination; builds the CSR of G and the CSC (= CSR of G^R,
+ * Alg 1 l.5 P:741, Alg 2 l.7 P:1043).  Vertex ids must be < n.
+ * Errors: CG_EINVAL (null pointers with m > 0, n <= 0, an id >= n, a weight 0),
+ *         CG_EOVERFLOW (see above), CG_ENOMEM, CG_ECUDA.  Synchronises `stream`.
+ */
+cg_status cg_graph_create(int device, int64_t n, int64_t m, const uint32_t* src, const uint32_t* dst,
+                          const uint32_t* w, void* stream, cg_graph* out);
+
+/* Release every device buffer owned by g (g may be NULL). */
+cg_status cg_graph_destroy(cg_graph g);
+
+/* Sizes of the canonical graph: n vertices, m edges, maximum weight.  Any output may be NULL. */
+cg_status cg_graph_info(cg_graph g, int64_t* n, int64_t* m, uint32_t* w_max);
+
+/* Copy the canonical CSR (transpose = 0) or CSC (transpose = 1) into caller device buffers:
+ * ptr int64[n+1], idx uint32[m] (destinations for CSR, sources for CSC), w uint32[m].
+ * Stream-ordered. */
+cg_status cg_graph_export(cg_graph g, int transpose, int64_t* ptr, uint32_t* idx, uint32_t* w, void* stream);
+
+/*
+ * Build the Core Graph CG(V, E_c) used by `kind` (Algorithm 1 P:727-786 or Algorithm 2
+ * P:1022-1085, see cg_cg_alg), from K hubs chosen by `policy` (`hubs`: host array of K
+ * ids, CG_HUBS_GIVEN only; `seed`: CG_HUBS_SAMPLED only).  connectivity != 0 applies
+ * Alg 1 l.8-12 (one out-edge for every vertex with outdeg > 0, reading Q8);
+ * the default (cg_build) applies it to Algorithm 1 CGs and not to Algorithm 2 CGs
+ * (reading Q11).  BFS and REACH share one general CG.  Rebuilding replaces the old CG.
+ * Errors: CG_EINVAL (K <= 0, K > n, bad policy / hubs), CG_ENOMEM, CG_ECUDA.
+ * Synchronises `stream`.
+ */
+cg_status cg_build(cg_graph g, cg_kind kind, int32_t K, cg_hub_policy policy, const uint32_t* hubs,
+                   uint64_t seed, void* stream);
+cg_status cg_build_ex(cg_graph g, cg_kind kind, int32_t K, cg_hub_policy policy, const uint32_t* hubs,
+                      uint64_t seed, cg_cg_alg alg, int32_t connectivity, void* stream);
+
+/* Core Graph sizes for `kind`: m_cg edges, K hubs (hubs: host buffer of >= K entries, may be NULL),
+ * build_ms = device time of the last cg_build for that kind.  CG_ENOCG if not built. */
+cg_status cg_core_info(cg_graph g, cg_kind kind, int64_t* m_cg, int32_t* K, uint32_t* hubs, float* build_ms);
+
+/* Copy the Core Graph's edge membership as flags (uint8[m], device, 1 = edge in E_c) in G's
+ * canonical CSR edge order.  Stream-ordered.  CG_ENOCG if not built. */
+cg_status cg_core_export(cg_graph g, cg_kind kind, uint8_t* flags, void* stream);
+
+/*
+ * Evaluate n_src vertex queries Q(s) of `kind`, writing Val(*) of query q to
+ * out[q*n .. q*n+n) (device, uint32 words; binary32 for VITERBI).  Unreached vertices hold
+ * InitVal, out[q*n + s] = SourceInitVal (reading Q1).  src: device array of n_src ids.
+ * mode: CG_MODE_2PHASE (Alg 3: init, phase 1 on CG, phase 2 on G from the impacted set) or
+ * CG_MODE_FULL.  The results of both modes are identical.
+ * p1_out (device, nullable): phase-1 values per query (2PHASE only), enables precise_p1.
+ * stats (host, nullable, n_src entries): per-query counters; if non-NULL the call
+ * synchronises `stream`, else it is fully asynchronous (one persistent kernel launch).
+ * Errors: CG_EINVAL, CG_ENOCG, CG_ENOMEM, CG_ECUDA, CG_EINTERNAL.
+ */
+cg_status cg_query(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode, void* out,
+                   cg_stats* stats, void* stream);
+cg_status cg_query_ex(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode, void* out,
+                      void* p1_out, cg_stats* stats, void* stream);
+
+/*
+ * End-to-end variant with HOST buffers: src (host, n_src ids) and out (host, n_src*n words).
+ * Copies sources host->device, runs the queries in device batches of `batch` (<= 0: auto)
+ * and streams each batch's values device->host while the next batch computes (two internal
+ * streams ordered after `stream`).  Synchronises `stream` before returning.
+ */
+cg_status cg_query_host(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode, void* out,
+                        int32_t batch, void* stream);
+
+/*
+ * Device twin of the seeded R-MAT input generator (gen/rmat.c defines it): edges
+ * [e0, e0+count) into device arrays src/dst/w.  tA/tAB/tABC are the integer quadrant
+ * thresholds floor(p*2^32).  Stream-ordered.
+ */
+cg_status cg_rmat_generate(uint64_t n, uint32_t tA, uint32_t tAB, uint32_t tABC, uint32_t w_max, uint64_t seed,
+                           int32_t permute, uint64_t e0, uint64_t count, uint32_t* src, uint32_t* dst, uint32_t* w,
+                           void* stream);
+
+/* Number of CUDA kernels this library has launched in this process (for launch accounting). */
+int64_t cg_kernel_launches(void);
+
+/* Human-readable name of a status code, and the thread-local detail of the last error. */
+const char* cg_status_string(cg_status s);
+const char* cg_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* CG_H */

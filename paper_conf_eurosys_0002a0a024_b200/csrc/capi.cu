@@ -1,0 +1,322 @@
+// capi.cu — the extern "C" boundary declared in include/cg.h.  Argument checking, error
+// translation (no exception crosses the ABI), allocator plumbing, and the host-buffer
+// end-to-end query path.  All compute happens in the kernels of the other .cu files.
+#include <cstring>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "graph.hpp"
+
+namespace cgb {
+
+std::atomic<int64_t> g_launches{0};
+
+namespace {
+cg_alloc_fn g_alloc = nullptr;
+cg_free_fn g_free = nullptr;
+void* g_ctx = nullptr;
+thread_local std::string g_err;
+}  // namespace
+
+void* dev_alloc(size_t bytes, cudaStream_t s) {
+    if (!bytes) return nullptr;
+    void* p = nullptr;
+    if (g_alloc) {
+        p = g_alloc(bytes, (void*)s, g_ctx);
+        if (!p) throw Error(CG_ENOMEM, "allocator callback failed for " + std::to_string(bytes) + " bytes");
+        return p;
+    }
+    cudaError_t e = cudaMalloc(&p, bytes);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        throw Error(CG_ENOMEM, "cudaMalloc(" + std::to_string(bytes) + "): " + cudaGetErrorString(e));
+    }
+    return p;
+}
+
+void dev_free(void* p, cudaStream_t s) {
+    if (!p) return;
+    if (g_free) g_free(p, (void*)s, g_ctx);
+    else {
+        cudaStreamSynchronize(s);
+        cudaFree(p);
+    }
+}
+
+}  // namespace cgb
+
+using namespace cgb;
+
+struct cg_graph_s {
+    Graph G;
+    cudaStream_t stream = nullptr;  // stream the graph's memory was allocated on
+};
+
+namespace capi_internal {
+
+template <typename F>
+cg_status guard(F&& f) {
+    try {
+        f();
+        return CG_OK;
+    } catch (const Error& e) {
+        g_err = e.what();
+        return e.code;
+    } catch (const std::bad_alloc&) {
+        g_err = "host allocation failed";
+        return CG_ENOMEM;
+    } catch (const std::exception& e) {
+        g_err = e.what();
+        return CG_EINTERNAL;
+    } catch (...) {
+        g_err = "unknown exception";
+        return CG_EINTERNAL;
+    }
+}
+
+inline cudaStream_t S(void* s) { return (cudaStream_t)s; }
+
+void check_kind(int kind) { CGB_CHECK(kind >= CG_SSSP && kind <= CG_REACH, CG_EINVAL, "bad cg_kind"); }
+
+void check_sources_host(const Graph& G, const uint32_t* src, int32_t n_src) {
+    for (int32_t i = 0; i < n_src; ++i) CGB_CHECK(src[i] < G.n, CG_EINVAL, "source id >= n");
+}
+
+__global__ void k_check_src(const uint32_t* __restrict__ src, int32_t n_src, uint32_t n, uint32_t* bad) {
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n_src; i += gridDim.x * blockDim.x)
+        if (src[i] >= n) atomicOr(bad, 1u);
+}
+
+void prepare_query(cg_graph g, int kind, int32_t n_src, int mode, const void* out, const uint32_t* src) {
+    CGB_CHECK(g != nullptr, CG_EINVAL, "null graph");
+    check_kind(kind);
+    CGB_CHECK(n_src >= 0, CG_EINVAL, "n_src < 0");
+    CGB_CHECK(mode == CG_MODE_2PHASE || mode == CG_MODE_FULL, CG_EINVAL, "bad cg_mode");
+    CGB_CHECK(n_src == 0 || (out && src), CG_EINVAL, "null src/out");
+    if (kind == CG_SSSP)
+        CGB_CHECK((uint64_t)(g->G.n - 1) * g->G.w_max < 0xFFFFFFFFull, CG_EOVERFLOW,
+                  "(n-1)*w_max >= 2^32-1: SSSP distances could wrap");
+    if (mode == CG_MODE_2PHASE)
+        CGB_CHECK(g->G.core[core_slot(kind)].built, CG_ENOCG, "cg_build has not been called for this kind");
+}
+
+}  // namespace capi_internal
+
+using namespace capi_internal;
+
+extern "C" {
+
+cg_status cg_set_allocator(cg_alloc_fn alloc, cg_free_fn free_fn, void* ctx) {
+    return guard([&] {
+        CGB_CHECK((alloc == nullptr) == (free_fn == nullptr), CG_EINVAL, "alloc and free must both be set or NULL");
+        g_alloc = alloc;
+        g_free = free_fn;
+        g_ctx = ctx;
+    });
+}
+
+cg_status cg_graph_create(int device, int64_t n, int64_t m, const uint32_t* src, const uint32_t* dst,
+                          const uint32_t* w, void* stream, cg_graph* out) {
+    return guard([&] {
+        CGB_CHECK(out != nullptr, CG_EINVAL, "null out");
+        *out = nullptr;
+        CGB_CHECK(n > 0, CG_EINVAL, "n must be > 0");
+        CGB_CHECK(m >= 0, CG_EINVAL, "m must be >= 0");
+        CGB_CHECK(m == 0 || (src && dst && w), CG_EINVAL, "null edge array");
+        CGB_CUDA(cudaSetDevice(device));
+        int coop = 0;
+        CGB_CUDA(cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, device));
+        CGB_CHECK(coop, CG_EUNSUPPORTED, "device does not support cooperative launch");
+        auto* h = new cg_graph_s();
+        try {
+            h->G.device = device;
+            h->stream = S(stream);
+            CGB_CUDA(cudaDeviceGetAttribute(&h->G.num_sms, cudaDevAttrMultiProcessorCount, device));
+            build_graph(h->G, n, m, src, dst, w, S(stream));
+        } catch (...) {
+            delete h;
+            throw;
+        }
+        *out = h;
+    });
+}
+
+cg_status cg_graph_destroy(cg_graph g) {
+    return guard([&] {
+        if (!g) return;
+        cudaSetDevice(g->G.device);
+        cudaStreamSynchronize(g->stream);
+        delete g;
+    });
+}
+
+cg_status cg_graph_info(cg_graph g, int64_t* n, int64_t* m, uint32_t* w_max) {
+    return guard([&] {
+        CGB_CHECK(g != nullptr, CG_EINVAL, "null graph");
+        if (n) *n = g->G.n;
+        if (m) *m = g->G.m;
+        if (w_max) *w_max = g->G.w_max;
+    });
+}
+
+cg_status cg_graph_export(cg_graph g, int transpose, int64_t* ptr, uint32_t* idx, uint32_t* w, void* stream) {
+    return guard([&] {
+        CGB_CHECK(g != nullptr, CG_EINVAL, "null graph");
+        CGB_CHECK(ptr && (g->G.m == 0 || (idx && w)), CG_EINVAL, "null output");
+        CGB_CUDA(cudaSetDevice(g->G.device));
+        export_adj(g->G, transpose ? g->G.gr : g->G.g, ptr, idx, w, S(stream));
+    });
+}
+
+cg_status cg_build_ex(cg_graph g, cg_kind kind, int32_t K, cg_hub_policy policy, const uint32_t* hubs, uint64_t seed,
+                      cg_cg_alg alg, int32_t connectivity, void* stream) {
+    return guard([&] {
+        CGB_CHECK(g != nullptr, CG_EINVAL, "null graph");
+        check_kind(kind);
+        CGB_CUDA(cudaSetDevice(g->G.device));
+        if (kind == CG_SSSP)
+            CGB_CHECK((uint64_t)(g->G.n - 1) * g->G.w_max < 0xFFFFFFFFull, CG_EOVERFLOW,
+                      "(n-1)*w_max >= 2^32-1: SSSP distances could wrap");
+        build_core(g->G, kind, K, policy, hubs, seed, alg, connectivity, S(stream));
+    });
+}
+
+cg_status cg_build(cg_graph g, cg_kind kind, int32_t K, cg_hub_policy policy, const uint32_t* hubs, uint64_t seed,
+                   void* stream) {
+    return cg_build_ex(g, kind, K, policy, hubs, seed, CG_ALG_AUTO, -1, stream);
+}
+
+cg_status cg_core_info(cg_graph g, cg_kind kind, int64_t* m_cg, int32_t* K, uint32_t* hubs, float* build_ms) {
+    return guard([&] {
+        CGB_CHECK(g != nullptr, CG_EINVAL, "null graph");
+        check_kind(kind);
+        const Core& C = g->G.core[core_slot(kind)];
+        CGB_CHECK(C.built, CG_ENOCG, "Core Graph not built for this kind");
+        if (m_cg) *m_cg = C.adj.m;
+        if (K) *K = (int32_t)C.hubs.size();
+        if (hubs) std::memcpy(hubs, C.hubs.data(), 4 * C.hubs.size());
+        if (build_ms) *build_ms = C.build_ms;
+    });
+}
+
+cg_status cg_core_export(cg_graph g, cg_kind kind, uint8_t* flags, void* stream) {
+    return guard([&] {
+        CGB_CHECK(g != nullptr && flags != nullptr, CG_EINVAL, "null argument");
+        check_kind(kind);
+        const Core& C = g->G.core[core_slot(kind)];
+        CGB_CHECK(C.built, CG_ENOCG, "Core Graph not built for this kind");
+        CGB_CUDA(cudaSetDevice(g->G.device));
+        if (g->G.m)
+            CGB_CUDA(cudaMemcpyAsync(flags, C.flags.get(), g->G.m, cudaMemcpyDeviceToDevice, S(stream)));
+    });
+}
+
+cg_status cg_query_ex(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode, void* out,
+                      void* p1_out, cg_stats* stats, void* stream) {
+    return guard([&] {
+        prepare_query(g, kind, n_src, mode, out, src);
+        if (n_src == 0) return;
+        Graph& G = g->G;
+        CGB_CUDA(cudaSetDevice(G.device));
+        if (stats) {  // validate sources on device (the call synchronises anyway)
+            DevBuf<uint32_t> bad(1, S(stream));
+            CGB_CUDA(cudaMemsetAsync(bad.get(), 0, 4, S(stream)));
+            CGB_LAUNCH(k_check_src, 1, 256, 0, S(stream), src, n_src, G.n, bad.get());
+            uint32_t hb = 0;
+            CGB_CUDA(cudaMemcpyAsync(&hb, bad.get(), 4, cudaMemcpyDeviceToHost, S(stream)));
+            CGB_CUDA(cudaStreamSynchronize(S(stream)));
+            CGB_CHECK(!hb, CG_EINVAL, "source id >= n");
+        }
+        const bool two = mode == CG_MODE_2PHASE;
+        QueryCall c{(int)kind, view(G.g), two ? view(G.core[core_slot(kind)].adj) : view(G.g), two ? 1 : 0, src,
+                    n_src, (uint32_t*)out, two ? (uint32_t*)p1_out : nullptr, stats != nullptr};
+        std::vector<cg_stats> st;
+        run_queries(G, c, S(stream), stats ? &st : nullptr);
+        if (stats) std::memcpy(stats, st.data(), sizeof(cg_stats) * (size_t)n_src);
+    });
+}
+
+cg_status cg_query(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode, void* out,
+                   cg_stats* stats, void* stream) {
+    return cg_query_ex(g, kind, src, n_src, mode, out, nullptr, stats, stream);
+}
+
+cg_status cg_query_host(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode, void* out,
+                        int32_t batch, void* stream) {
+    return guard([&] {
+        prepare_query(g, kind, n_src, mode, out, src);
+        if (n_src == 0) return;
+        Graph& G = g->G;
+        check_sources_host(G, src, n_src);
+        CGB_CUDA(cudaSetDevice(G.device));
+        cudaStream_t s = S(stream);
+        const size_t row = (size_t)G.n * 4;
+        if (batch <= 0) {  // ~256 MiB of results per batch, at least 1 query
+            size_t b = ((size_t)256 << 20) / (row ? row : 1);
+            batch = (int32_t)(b < 1 ? 1 : (b > (size_t)n_src ? (size_t)n_src : b));
+        }
+        if (batch > n_src) batch = n_src;
+        DevBuf<uint32_t> dsrc((size_t)n_src, s);
+        CGB_CUDA(cudaMemcpyAsync(dsrc.get(), src, 4ull * n_src, cudaMemcpyHostToDevice, s));
+        // two result slots: batch b computes on `s` into slot b%2 while batch b-1 drains on `cp`
+        DevBuf<uint32_t> slot[2];
+        slot[0].alloc((size_t)batch * G.n, s);
+        if (n_src > batch) slot[1].alloc((size_t)batch * G.n, s);
+        cudaStream_t cp;
+        CGB_CUDA(cudaStreamCreateWithFlags(&cp, cudaStreamNonBlocking));
+        cudaEvent_t done[2], drained[2];
+        for (int i = 0; i < 2; ++i) {
+            CGB_CUDA(cudaEventCreateWithFlags(&done[i], cudaEventDisableTiming));
+            CGB_CUDA(cudaEventCreateWithFlags(&drained[i], cudaEventDisableTiming));
+        }
+        const bool two = mode == CG_MODE_2PHASE;
+        int b = 0;
+        for (int32_t q0 = 0; q0 < n_src; q0 += batch, ++b) {
+            const int32_t nq = (n_src - q0) < batch ? (n_src - q0) : batch;
+            const int k = b & 1;
+            if (b >= 2) CGB_CUDA(cudaStreamWaitEvent(s, drained[k], 0));
+            QueryCall c{(int)kind, view(G.g), two ? view(G.core[core_slot(kind)].adj) : view(G.g), two ? 1 : 0,
+                        dsrc.get() + q0, nq, slot[k].get(), nullptr, false};
+            run_queries(G, c, s, nullptr);
+            CGB_CUDA(cudaEventRecord(done[k], s));
+            CGB_CUDA(cudaStreamWaitEvent(cp, done[k], 0));
+            CGB_CUDA(cudaMemcpyAsync((uint32_t*)out + (size_t)q0 * G.n, slot[k].get(), (size_t)nq * row,
+                                     cudaMemcpyDeviceToHost, cp));
+            CGB_CUDA(cudaEventRecord(drained[k], cp));
+        }
+        CGB_CUDA(cudaStreamSynchronize(cp));
+        CGB_CUDA(cudaStreamSynchronize(s));
+        for (int i = 0; i < 2; ++i) {
+            cudaEventDestroy(done[i]);
+            cudaEventDestroy(drained[i]);
+        }
+        cudaStreamDestroy(cp);
+    });
+}
+
+cg_status cg_rmat_generate(uint64_t n, uint32_t tA, uint32_t tAB, uint32_t tABC, uint32_t w_max, uint64_t seed,
+                           int32_t permute, uint64_t e0, uint64_t count, uint32_t* src, uint32_t* dst, uint32_t* w,
+                           void* stream) {
+    return guard([&] { rmat_generate(n, tA, tAB, tABC, w_max, seed, permute, e0, count, src, dst, w, S(stream)); });
+}
+
+int64_t cg_kernel_launches(void) { return g_launches.load(); }
+
+const char* cg_status_string(cg_status s) {
+    switch (s) {
+    case CG_OK: return "CG_OK";
+    case CG_EINVAL: return "CG_EINVAL";
+    case CG_ENOMEM: return "CG_ENOMEM";
+    case CG_ECUDA: return "CG_ECUDA";
+    case CG_ENOCG: return "CG_ENOCG";
+    case CG_EOVERFLOW: return "CG_EOVERFLOW";
+    case CG_EUNSUPPORTED: return "CG_EUNSUPPORTED";
+    case CG_EINTERNAL: return "CG_EINTERNAL";
+    }
+    return "CG_UNKNOWN";
+}
+
+const char* cg_last_error(void) { return g_err.c_str(); }
+
+}  // extern "C"

@@ -1,0 +1,127 @@
+// common.cuh — internal helpers of the B200 Core Graph library (not part of the ABI).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <atomic>
+#include <stdexcept>
+#include <string>
+
+#include "../../include/cg.h"
+
+namespace cgb {
+
+// ---------------------------------------------------------------- errors
+struct Error : std::runtime_error {
+    cg_status code;
+    Error(cg_status c, const std::string& msg) : std::runtime_error(msg), code(c) {}
+};
+
+#define CGB_CUDA(call)                                                                         \
+    do {                                                                                       \
+        cudaError_t _e = (call);                                                               \
+        if (_e != cudaSuccess)                                                                 \
+            throw ::cgb::Error(_e == cudaErrorMemoryAllocation ? CG_ENOMEM : CG_ECUDA,         \
+                               std::string(#call) + ": " + cudaGetErrorString(_e));            \
+    } while (0)
+
+#define CGB_CHECK(cond, code, msg)                                                             \
+    do {                                                                                       \
+        if (!(cond)) throw ::cgb::Error((code), (msg));                                        \
+    } while (0)
+
+// ---------------------------------------------------------------- launch accounting
+extern std::atomic<int64_t> g_launches;
+inline void count_launch(int64_t k = 1) { g_launches.fetch_add(k, std::memory_order_relaxed); }
+
+#define CGB_LAUNCH(kernel, grid, block, smem, stream, ...)                                      \
+    do {                                                                                       \
+        kernel<<<(grid), (block), (smem), (stream)>>>(__VA_ARGS__);                            \
+        ::cgb::count_launch();                                                                 \
+        CGB_CUDA(cudaGetLastError());                                                          \
+    } while (0)
+
+// ---------------------------------------------------------------- memory
+void* dev_alloc(size_t bytes, cudaStream_t s);
+void dev_free(void* p, cudaStream_t s);
+
+template <typename T>
+struct DevBuf {
+    T* p = nullptr;
+    size_t n = 0;
+    cudaStream_t s = nullptr;
+    DevBuf() = default;
+    DevBuf(size_t count, cudaStream_t st) { alloc(count, st); }
+    DevBuf(const DevBuf&) = delete;
+    DevBuf& operator=(const DevBuf&) = delete;
+    DevBuf(DevBuf&& o) noexcept : p(o.p), n(o.n), s(o.s) { o.p = nullptr; o.n = 0; }
+    DevBuf& operator=(DevBuf&& o) noexcept {
+        if (this != &o) { reset(); p = o.p; n = o.n; s = o.s; o.p = nullptr; o.n = 0; }
+        return *this;
+    }
+    ~DevBuf() { reset(); }
+    void alloc(size_t count, cudaStream_t st) {
+        reset();
+        s = st;
+        n = count;
+        p = count ? static_cast<T*>(dev_alloc(count * sizeof(T), st)) : nullptr;
+    }
+    void reset() {
+        if (p) dev_free(p, s);
+        p = nullptr;
+        n = 0;
+    }
+    T* get() const { return p; }
+    size_t bytes() const { return n * sizeof(T); }
+};
+
+// ---------------------------------------------------------------- device helpers
+__device__ __forceinline__ uint32_t ld_cg(const uint32_t* p) {
+    uint32_t v;
+    asm volatile("ld.global.cg.u32 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ unsigned long long ld_cg64(const unsigned long long* p) {
+    unsigned long long v;
+    asm volatile("ld.global.cg.u64 %0, [%1];" : "=l"(v) : "l"(p));
+    return v;
+}
+// streaming read-only edge words: no L1 allocation, evict-first L2 policy
+__device__ __forceinline__ uint64_t policy_evict_first() {
+    uint64_t p;
+    asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ uint32_t ld_stream(const uint32_t* p) {
+    uint32_t v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;"
+                 : "=r"(v)
+                 : "l"(p), "l"(policy_evict_first()));
+    return v;
+}
+__device__ __forceinline__ uint4 ld_stream4(const uint4* p) {
+    uint4 v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+                 : "l"(p), "l"(policy_evict_first()));
+    return v;
+}
+__device__ __forceinline__ uint2 ld_stream2(const uint2* p) {
+    uint2 v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.u32 {%0,%1}, [%2], %3;"
+                 : "=r"(v.x), "=r"(v.y)
+                 : "l"(p), "l"(policy_evict_first()));
+    return v;
+}
+__device__ __forceinline__ uint32_t ld_ro(const uint32_t* p) { return __ldg(p); }
+
+__device__ __forceinline__ void red_or(uint32_t* p, uint32_t v) {
+    asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+__device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31u; }
+
+inline int ceil_div(int64_t a, int64_t b) { return (int)((a + b - 1) / b); }
+
+}  // namespace cgb

@@ -1,0 +1,436 @@
+// core_graph.cu — Core Graph construction on the GPU (SURVEY §8(a) rows a3-a7, a5').
+//
+//   a3 hub selection: K highest total-degree vertices, ties to the smaller id (P:464-466,
+//      P:1669-1677, reading Q7), or K sampled / given ids (north_star, reading D2).
+//   a4 Identify queries (Alg 1 l.3-7): forward Q(h) on G and backward Q(h) on
+//      G^R for every hub, run by the same persistent relaxation kernel (FULL mode).
+//   a5 tight-edge marking (Alg 1 l.15-25) evaluated directly on G's CSR rows:
+//      forward  e(u,v): reached_f(u) && Val_f(u) (+) w == Val_f(v)
+//      backward e(u,v): reached_b(v) && Val_b(v) (+) w == Val_b(u)   (the G^R edge v->u,
+//      reversed back into G's orientation, l.21), so no edge-id map is needed.
+//   a5' Algorithm 2 for BFS / REACH: exact emulation of the sequential FIFO
+//      traversals with a shared Qid[] — level-synchronous, each newly labeled vertex's
+//      discovering edge is the minimum (FIFO rank of parent, position in parent's row),
+//      which is the edge the FIFO examines first; the next level is ordered by that key.
+//   a6 connectivity edges (Alg 1 l.8-12; reading Q8).
+//   a7 stream compaction of the flagged edges into the CG's CSR.
+#include <cub/device/device_scan.cuh>
+
+#include <chrono>
+#include <cstring>
+
+#include "graph.hpp"
+
+namespace cgb {
+
+namespace {
+
+constexpr int TB = 256;
+constexpr uint32_t FULLM = 0xffffffffu;
+
+inline int grid_rows(uint64_t rows) {
+    uint64_t warps = rows;
+    uint64_t g = (warps * 32 + TB - 1) / TB;
+    if (g > 65536) g = 65536;
+    return (int)(g ? g : 1);
+}
+
+template <int KIND> struct K;
+template <> struct K<CG_SSSP> {
+    static constexpr uint32_t INIT = 0xffffffffu;
+    __device__ static uint32_t ext(uint32_t a, uint32_t w) { return a + w; }
+};
+template <> struct K<CG_SSWP> {
+    static constexpr uint32_t INIT = 0u;
+    __device__ static uint32_t ext(uint32_t a, uint32_t w) { return min(a, w); }
+};
+template <> struct K<CG_SSNP> {
+    static constexpr uint32_t INIT = 0xffffffffu;
+    __device__ static uint32_t ext(uint32_t a, uint32_t w) { return max(a, w); }
+};
+template <> struct K<CG_VITERBI> {
+    static constexpr uint32_t INIT = 0u;
+    __device__ static uint32_t ext(uint32_t a, uint32_t w) {
+        return __float_as_uint(__fdiv_rn(__uint_as_float(a), __uint2float_rn(w)));
+    }
+};
+template <> struct K<CG_BFS> {
+    static constexpr uint32_t INIT = 0xffffffffu;
+    __device__ static uint32_t ext(uint32_t a, uint32_t) { return a + 1u; }
+};
+template <> struct K<CG_REACH> {
+    static constexpr uint32_t INIT = 0u;
+    __device__ static uint32_t ext(uint32_t a, uint32_t) { return a; }
+};
+
+__device__ __forceinline__ void edge_at(const GraphView& g, uint32_t e, uint32_t dbits, uint32_t& d, uint32_t& w) {
+    if (g.adj) {
+        uint32_t x = g.adj[e];
+        d = dbits >= 32 ? x : (x & ((1u << dbits) - 1u));
+        w = (x >> dbits) + 1u;
+    } else {
+        uint2 x = g.adjw[e];
+        d = x.x;
+        w = x.y;
+    }
+}
+
+// ---------------------------------------------------------------- a3: hubs
+__global__ void k_degree_key_max(uint32_t n, const uint32_t* __restrict__ ptr, const uint32_t* __restrict__ rptr,
+                                 const unsigned long long* __restrict__ bound, unsigned long long* __restrict__ out) {
+    const unsigned long long lim = *bound;
+    unsigned long long best = 0;
+    for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x) {
+        const unsigned long long deg = (unsigned long long)(ptr[v + 1] - ptr[v]) + (rptr[v + 1] - rptr[v]);
+        const unsigned long long key = (deg << 32) | (0xffffffffull - v);  // larger degree, then smaller id
+        if (key < lim && key > best) best = key;
+    }
+    for (int o = 16; o > 0; o >>= 1) {
+        unsigned long long y = __shfl_xor_sync(FULLM, best, o);
+        best = y > best ? y : best;
+    }
+    if ((threadIdx.x & 31) == 0 && best) atomicMax(out, best);
+}
+
+// ---------------------------------------------------------------- a5: Alg 1 marking
+// Warp per row u of G; hubs [0, nh) of the current group; valf/valb: nh x n values.
+template <int KIND>
+__global__ void k_mark_tight(uint32_t n, GraphView g, uint32_t dbits, int nh, const uint32_t* __restrict__ valf,
+                             const uint32_t* __restrict__ valb, uint8_t* __restrict__ flags) {
+    using O = K<KIND>;
+    const uint32_t lane = threadIdx.x & 31;
+    const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
+    for (uint64_t u = blockIdx.x * (uint64_t)(blockDim.x / 32) + (threadIdx.x >> 5); u < n; u += nw) {
+        const uint32_t r0 = g.ptr[u], r1 = g.ptr[u + 1];
+        for (uint32_t e = r0 + lane; e < r1; e += 32) {
+            uint32_t v, w;
+            edge_at(g, e, dbits, v, w);
+            bool tight = false;
+            for (int k = 0; k < nh && !tight; ++k) {
+                const uint32_t* vf = valf + (size_t)k * n;
+                const uint32_t* vb = valb + (size_t)k * n;
+                const uint32_t fu = vf[u];
+                if (fu != O::INIT && O::ext(fu, w) == vf[v]) tight = true;   // l.16-19, d == f
+                const uint32_t bv = vb[v];
+                if (bv != O::INIT && O::ext(bv, w) == vb[u]) tight = true;   // l.16-21, d == b
+            }
+            if (tight) flags[e] = 1;
+        }
+    }
+}
+
+// ---------------------------------------------------------------- a6: connectivity
+// kind_sel: 0 = min weight (SSSP/SSNP/Viterbi), 1 = max weight (SSWP), 2 = first edge.
+__global__ void k_connectivity(uint32_t n, GraphView g, uint32_t dbits, int kind_sel, uint8_t* __restrict__ flags) {
+    const uint32_t lane = threadIdx.x & 31;
+    const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
+    for (uint64_t u = blockIdx.x * (uint64_t)(blockDim.x / 32) + (threadIdx.x >> 5); u < n; u += nw) {
+        const uint32_t r0 = g.ptr[u], r1 = g.ptr[u + 1];
+        if (r0 == r1) continue;
+        bool any = false;
+        unsigned long long best = ~0ull;
+        for (uint32_t e = r0 + lane; e < r1; e += 32) {
+            any |= flags[e] != 0;
+            uint32_t v, w;
+            edge_at(g, e, dbits, v, w);
+            const uint32_t wk = kind_sel == 0 ? w : (kind_sel == 1 ? ~w : 0u);
+            const unsigned long long key = ((unsigned long long)wk << 32) | (e - r0);
+            best = key < best ? key : best;
+        }
+        if (__any_sync(FULLM, any)) continue;
+        for (int o = 16; o > 0; o >>= 1) {
+            unsigned long long y = __shfl_xor_sync(FULLM, best, o);
+            best = y < best ? y : best;
+        }
+        if (lane == 0) flags[r0 + (uint32_t)best] = 1;
+    }
+}
+
+// ---------------------------------------------------------------- a7: compaction
+__global__ void k_row_count(uint32_t n, const uint32_t* __restrict__ ptr, const uint8_t* __restrict__ flags,
+                            uint32_t* __restrict__ cnt) {
+    const uint32_t lane = threadIdx.x & 31;
+    const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
+    for (uint64_t u = blockIdx.x * (uint64_t)(blockDim.x / 32) + (threadIdx.x >> 5); u <= n; u += nw) {
+        if (u == n) { if (lane == 0) cnt[n] = 0; continue; }
+        uint32_t c = 0;
+        for (uint32_t e = ptr[u] + lane; e < ptr[u + 1]; e += 32) c += flags[e] != 0;
+        for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(FULLM, c, o);
+        if (lane == 0) cnt[u] = c;
+    }
+}
+
+__global__ void k_scatter_core(uint32_t n, const uint32_t* __restrict__ ptr, const uint8_t* __restrict__ flags,
+                               const uint32_t* __restrict__ cptr, const uint32_t* __restrict__ adj,
+                               const uint2* __restrict__ adjw, uint32_t* __restrict__ cadj, uint2* __restrict__ cadjw) {
+    const uint32_t lane = threadIdx.x & 31;
+    const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
+    for (uint64_t u = blockIdx.x * (uint64_t)(blockDim.x / 32) + (threadIdx.x >> 5); u < n; u += nw) {
+        uint32_t o = cptr[u];
+        const uint32_t r0 = ptr[u], r1 = ptr[u + 1];
+        for (uint32_t b = r0; b < r1; b += 32) {
+            const uint32_t e = b + lane;
+            const bool f = e < r1 && flags[e];
+            const uint32_t bal = __ballot_sync(FULLM, f);
+            if (f) {
+                const uint32_t p = o + __popc(bal & ((1u << lane) - 1u));
+                if (adj) cadj[p] = adj[e]; else cadjw[p] = adjw[e];
+            }
+            o += __popc(bal);
+        }
+    }
+}
+
+// ---------------------------------------------------------------- a5': Alg 2
+// Expand level L (FIFO order = list order) of a traversal labeled `lab`.
+template <bool REV>
+__global__ void k_alg2_expand(GraphView g, uint32_t dbits, const uint32_t* __restrict__ L, uint32_t nl,
+                              const uint32_t* __restrict__ qid, uint32_t lab, unsigned long long* __restrict__ key,
+                              uint8_t* __restrict__ flags, const uint32_t* __restrict__ reid) {
+    const uint32_t lane = threadIdx.x & 31;
+    const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
+    for (uint64_t r = blockIdx.x * (uint64_t)(blockDim.x / 32) + (threadIdx.x >> 5); r < nl; r += nw) {
+        const uint32_t u = L[r];
+        const uint32_t r0 = g.ptr[u], r1 = g.ptr[u + 1];
+        for (uint32_t e = r0 + lane; e < r1; e += 32) {
+            uint32_t v, w;
+            edge_at(g, e, dbits, v, w);
+            const uint32_t q = qid[v];
+            if (q == lab) continue;                        // l.16: Qid(v) == s -> skip
+            if (q == 0)                                    // l.19: first examiner in FIFO order wins
+                atomicMin(key + v, ((unsigned long long)r << 32) | (e - r0));
+            else                                           // l.18: add e(u,v), v labeled elsewhere
+                flags[REV ? reid[e] : e] = 1;
+        }
+    }
+}
+
+__device__ __forceinline__ bool alg2_winner(const uint32_t* qid, const unsigned long long* key, uint32_t v, uint64_t r,
+                                            uint32_t j) {
+    return qid[v] == 0 && key[v] == ((((unsigned long long)r) << 32) | j);
+}
+
+template <bool EMIT, bool REV>
+__global__ void k_alg2_winners(GraphView g, uint32_t dbits, const uint32_t* __restrict__ L, uint32_t nl, uint32_t* qid,
+                               uint32_t lab, unsigned long long* key, uint32_t* __restrict__ cnt,
+                               const uint32_t* __restrict__ base, uint32_t* __restrict__ next,
+                               uint8_t* __restrict__ flags, const uint32_t* __restrict__ reid) {
+    const uint32_t lane = threadIdx.x & 31;
+    const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
+    for (uint64_t r = blockIdx.x * (uint64_t)(blockDim.x / 32) + (threadIdx.x >> 5); r < nl; r += nw) {
+        const uint32_t u = L[r];
+        const uint32_t r0 = g.ptr[u], r1 = g.ptr[u + 1];
+        uint32_t o = EMIT ? base[r] : 0u;
+        for (uint32_t b = r0; b < r1; b += 32) {
+            const uint32_t e = b + lane;
+            uint32_t v = 0, w;
+            bool win = false;
+            if (e < r1) {
+                edge_at(g, e, dbits, v, w);
+                win = alg2_winner(qid, key, v, r, e - r0);
+            }
+            const uint32_t bal = __ballot_sync(FULLM, win);
+            if (EMIT && win) {
+                next[o + __popc(bal & ((1u << lane) - 1u))] = v;   // l.20 Fifo.push(v)
+                flags[REV ? reid[e] : e] = 1;                      // l.18 add e(u,v)
+            }
+            o += __popc(bal);
+            __syncwarp();
+            if (EMIT && win) {                                     // l.21 Qid(v) <- s
+                qid[v] = lab;
+                key[v] = ~0ull;
+            }
+        }
+        if (!EMIT && lane == 0) cnt[r] = o;
+    }
+}
+
+void exclusive_sum(const uint32_t* in, uint32_t* out, uint64_t m, cudaStream_t s) {
+    size_t tmp = 0;
+    CGB_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, in, out, (int64_t)m, s));
+    DevBuf<uint8_t> t(tmp, s);
+    CGB_CUDA(cub::DeviceScan::ExclusiveSum(t.get(), tmp, in, out, (int64_t)m, s));
+    count_launch(2);
+}
+
+std::vector<uint32_t> select_hubs(Graph& G, int32_t K, int policy, const uint32_t* given, uint64_t seed,
+                                  cudaStream_t s) {
+    std::vector<uint32_t> hubs;
+    if (policy == CG_HUBS_GIVEN) {
+        CGB_CHECK(given != nullptr, CG_EINVAL, "CG_HUBS_GIVEN needs a host hub array");
+        for (int k = 0; k < K; ++k) {
+            CGB_CHECK(given[k] < G.n, CG_EINVAL, "hub id >= n");
+            hubs.push_back(given[k]);
+        }
+        return hubs;
+    }
+    if (policy == CG_HUBS_SAMPLED) {
+        // uniform over vertices with outdeg > 0, distinct, splitmix64(seed + i) draws
+        std::vector<uint32_t> ptr(G.n + 1);
+        CGB_CUDA(cudaMemcpyAsync(ptr.data(), G.g.ptr.get(), 4ull * (G.n + 1), cudaMemcpyDeviceToHost, s));
+        CGB_CUDA(cudaStreamSynchronize(s));
+        std::vector<uint32_t> cand;
+        for (uint32_t v = 0; v < G.n; ++v)
+            if (ptr[v + 1] > ptr[v]) cand.push_back(v);
+        CGB_CHECK((int64_t)cand.size() >= K, CG_EINVAL, "fewer than K vertices with outdeg > 0");
+        std::vector<uint8_t> taken(cand.size(), 0);
+        for (uint64_t i = 0; (int)hubs.size() < K; ++i) {
+            uint64_t x = seed + i * 0x9E3779B97F4A7C15ull;
+            x = (x ^ (x >> 30)) * 0xBF58476D1CE4E5B9ull;
+            x = (x ^ (x >> 27)) * 0x94D049BB133111EBull;
+            x ^= x >> 31;
+            const uint64_t j = x % cand.size();
+            if (!taken[j]) { taken[j] = 1; hubs.push_back(cand[j]); }
+        }
+        return hubs;
+    }
+    CGB_CHECK(policy == CG_HUBS_TOPDEG, CG_EINVAL, "bad hub policy");
+    DevBuf<unsigned long long> keys(K + 1, s);
+    const unsigned long long top = ~0ull;
+    CGB_CUDA(cudaMemsetAsync(keys.get(), 0, (K + 1) * 8ull, s));
+    CGB_CUDA(cudaMemcpyAsync(keys.get(), &top, 8, cudaMemcpyHostToDevice, s));
+    for (int k = 0; k < K; ++k)
+        CGB_LAUNCH(k_degree_key_max, 296, TB, 0, s, G.n, G.g.ptr.get(), G.gr.ptr.get(), keys.get() + k,
+                   keys.get() + k + 1);
+    std::vector<unsigned long long> h(K + 1);
+    CGB_CUDA(cudaMemcpyAsync(h.data(), keys.get(), (K + 1) * 8ull, cudaMemcpyDeviceToHost, s));
+    CGB_CUDA(cudaStreamSynchronize(s));
+    for (int k = 1; k <= K; ++k) hubs.push_back((uint32_t)(0xffffffffull - (h[k] & 0xffffffffull)));
+    return hubs;
+}
+
+template <int KIND>
+void mark_group(Graph& G, int nh, const uint32_t* vf, const uint32_t* vb, uint8_t* flags, cudaStream_t s) {
+    CGB_LAUNCH(k_mark_tight<KIND>, grid_rows(G.n), TB, 0, s, G.n, view(G.g), G.dbits, nh, vf, vb, flags);
+}
+
+void alg1(Graph& G, int kind, const std::vector<uint32_t>& hubs, uint8_t* flags, cudaStream_t s) {
+    const int K = (int)hubs.size();
+    const int group = K < 16 ? K : 16;
+    DevBuf<uint32_t> hsrc(K, s);
+    CGB_CUDA(cudaMemcpyAsync(hsrc.get(), hubs.data(), 4ull * K, cudaMemcpyHostToDevice, s));
+    DevBuf<uint32_t> vf((size_t)group * G.n, s), vb((size_t)group * G.n, s);
+    for (int k0 = 0; k0 < K; k0 += group) {
+        const int nh = (K - k0) < group ? (K - k0) : group;
+        QueryCall f{kind, view(G.g), view(G.g), 0, hsrc.get() + k0, nh, vf.get(), nullptr, false};
+        run_queries(G, f, s, nullptr);                   // Alg 1 l.4: Identify(G, forward)
+        QueryCall b{kind, view(G.gr), view(G.gr), 0, hsrc.get() + k0, nh, vb.get(), nullptr, false};
+        run_queries(G, b, s, nullptr);                   // Alg 1 l.5: Identify(G^R, backward)
+        switch (kind) {
+        case CG_SSSP: mark_group<CG_SSSP>(G, nh, vf.get(), vb.get(), flags, s); break;
+        case CG_SSWP: mark_group<CG_SSWP>(G, nh, vf.get(), vb.get(), flags, s); break;
+        case CG_SSNP: mark_group<CG_SSNP>(G, nh, vf.get(), vb.get(), flags, s); break;
+        case CG_VITERBI: mark_group<CG_VITERBI>(G, nh, vf.get(), vb.get(), flags, s); break;
+        case CG_BFS: mark_group<CG_BFS>(G, nh, vf.get(), vb.get(), flags, s); break;
+        case CG_REACH: mark_group<CG_REACH>(G, nh, vf.get(), vb.get(), flags, s); break;
+        }
+    }
+}
+
+void alg2(Graph& G, const std::vector<uint32_t>& hubs, uint8_t* flags, cudaStream_t s) {
+    const uint32_t n = G.n;
+    DevBuf<uint32_t> qid(n, s), la(n + 1, s), lb(n + 1, s), cnt(n + 1, s), base(n + 1, s);
+    DevBuf<unsigned long long> key(n, s);
+    CGB_CUDA(cudaMemsetAsync(qid.get(), 0, 4ull * n, s));
+    CGB_CUDA(cudaMemsetAsync(key.get(), 0xff, 8ull * n, s));
+    for (size_t k = 0; k < hubs.size(); ++k) {               // Alg 2 l.5
+        const uint32_t lab = (uint32_t)k + 1;                 // reading Q10
+        for (int dir = 0; dir < 2; ++dir) {                   // l.6 on G, l.7 on G^R
+            const GraphView g = dir == 0 ? view(G.g) : view(G.gr);
+            uint32_t* L = la.get();
+            uint32_t* N = lb.get();
+            uint32_t nl = 1;
+            CGB_CUDA(cudaMemcpyAsync(L, &hubs[k], 4, cudaMemcpyHostToDevice, s));   // l.12
+            while (nl) {                                                          // l.13
+                const int grid = grid_rows(nl);
+                if (dir == 0) {
+                    CGB_LAUNCH(k_alg2_expand<false>, grid, TB, 0, s, g, G.dbits, L, nl, qid.get(), lab, key.get(),
+                               flags, (const uint32_t*)nullptr);
+                    CGB_LAUNCH((k_alg2_winners<false, false>), grid, TB, 0, s, g, G.dbits, L, nl, qid.get(), lab,
+                               key.get(), cnt.get(), (const uint32_t*)nullptr, (uint32_t*)nullptr, flags,
+                               (const uint32_t*)nullptr);
+                } else {
+                    CGB_LAUNCH(k_alg2_expand<true>, grid, TB, 0, s, g, G.dbits, L, nl, qid.get(), lab, key.get(),
+                               flags, G.reid.get());
+                    CGB_LAUNCH((k_alg2_winners<false, true>), grid, TB, 0, s, g, G.dbits, L, nl, qid.get(), lab,
+                               key.get(), cnt.get(), (const uint32_t*)nullptr, (uint32_t*)nullptr, flags,
+                               G.reid.get());
+                }
+                CGB_CUDA(cudaMemsetAsync(cnt.get() + nl, 0, 4, s));
+                exclusive_sum(cnt.get(), base.get(), (uint64_t)nl + 1, s);
+                uint32_t total = 0;
+                CGB_CUDA(cudaMemcpyAsync(&total, base.get() + nl, 4, cudaMemcpyDeviceToHost, s));
+                CGB_CUDA(cudaStreamSynchronize(s));
+                if (total) {
+                    if (dir == 0)
+                        CGB_LAUNCH((k_alg2_winners<true, false>), grid, TB, 0, s, g, G.dbits, L, nl, qid.get(), lab,
+                                   key.get(), cnt.get(), base.get(), N, flags, (const uint32_t*)nullptr);
+                    else
+                        CGB_LAUNCH((k_alg2_winners<true, true>), grid, TB, 0, s, g, G.dbits, L, nl, qid.get(), lab,
+                                   key.get(), cnt.get(), base.get(), N, flags, G.reid.get());
+                }
+                uint32_t* t = L; L = N; N = t;
+                nl = total;
+            }
+        }
+    }
+}
+
+}  // namespace
+
+void build_core(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs_in, uint64_t seed, int alg,
+                int connectivity, cudaStream_t s) {
+    CGB_CHECK(kind >= 0 && kind <= CG_REACH, CG_EINVAL, "bad kind");
+    CGB_CHECK(K > 0 && (uint32_t)K <= G.n, CG_EINVAL, "K must be in [1, n]");
+    if (alg == CG_ALG_AUTO) alg = (kind == CG_BFS || kind == CG_REACH) ? CG_ALG_GENERAL : CG_ALG_SPECIALIZED;
+    CGB_CHECK(alg == CG_ALG_SPECIALIZED || alg == CG_ALG_GENERAL, CG_EINVAL, "bad CG algorithm");
+    if (connectivity < 0) connectivity = (alg == CG_ALG_SPECIALIZED) ? 1 : 0;
+
+    cudaEvent_t e0, e1;
+    CGB_CUDA(cudaEventCreate(&e0));
+    CGB_CUDA(cudaEventCreate(&e1));
+    CGB_CUDA(cudaEventRecord(e0, s));
+
+    std::vector<uint32_t> hubs = select_hubs(G, K, policy, hubs_in, seed, s);
+    Core& C = G.core[core_slot(kind)];
+    C.built = false;
+    C.flags.alloc(G.m ? G.m : 1, s);
+    CGB_CUDA(cudaMemsetAsync(C.flags.get(), 0, C.flags.bytes(), s));
+    if (G.m) {
+        if (alg == CG_ALG_SPECIALIZED) alg1(G, kind, hubs, C.flags.get(), s);
+        else alg2(G, hubs, C.flags.get(), s);
+        if (connectivity) {
+            const int sel = (kind == CG_SSWP) ? 1 : ((kind == CG_BFS || kind == CG_REACH) ? 2 : 0);
+            CGB_LAUNCH(k_connectivity, grid_rows(G.n), TB, 0, s, G.n, view(G.g), G.dbits, sel, C.flags.get());
+        }
+    }
+    // a7: compaction into the CG's CSR
+    DevBuf<uint32_t> cnt(G.n + 1, s);
+    C.adj.n = G.n;
+    C.adj.ptr.alloc(G.n + 1, s);
+    CGB_LAUNCH(k_row_count, grid_rows(G.n + 1), TB, 0, s, G.n, G.g.ptr.get(), C.flags.get(), cnt.get());
+    exclusive_sum(cnt.get(), C.adj.ptr.get(), (uint64_t)G.n + 1, s);
+    uint32_t mcg = 0;
+    CGB_CUDA(cudaMemcpyAsync(&mcg, C.adj.ptr.get() + G.n, 4, cudaMemcpyDeviceToHost, s));
+    CGB_CUDA(cudaStreamSynchronize(s));
+    C.adj.m = mcg;
+    C.adj.adj.reset();
+    C.adj.adjw.reset();
+    if (G.packed) C.adj.adj.alloc(mcg ? mcg : 1, s); else C.adj.adjw.alloc(mcg ? mcg : 1, s);
+    CGB_LAUNCH(k_scatter_core, grid_rows(G.n), TB, 0, s, G.n, G.g.ptr.get(), C.flags.get(), C.adj.ptr.get(),
+               G.g.adj.get(), G.g.adjw.get(), C.adj.adj.get(), C.adj.adjw.get());
+    build_big_bitmap(C.adj, s);
+    CGB_CUDA(cudaEventRecord(e1, s));
+    CGB_CUDA(cudaEventSynchronize(e1));
+    float ms = 0.f;
+    CGB_CUDA(cudaEventElapsedTime(&ms, e0, e1));
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    C.hubs = hubs;
+    C.alg = alg;
+    C.connectivity = connectivity;
+    C.build_ms = ms;
+    C.built = true;
+}
+
+}  // namespace cgb

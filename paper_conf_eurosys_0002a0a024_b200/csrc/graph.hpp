@@ -1,0 +1,102 @@
+// graph.hpp — device-resident graph store (G, G^R, Core Graphs) and query workspace.
+#pragma once
+
+#include <vector>
+
+#include "common.cuh"
+
+namespace cgb {
+
+// Rows with at least kBigThreshold out-edges are split into kChunk-edge pieces that all
+// warps of the grid share (the "CTA-per-high-degree" tier, generalised to multi-CTA).
+constexpr uint32_t kBigThreshold = 2048;
+constexpr uint32_t kChunk = 512;
+
+// Out-edge structure in the engine's HBM layout:
+//   ptr   u32[n+1]  row offsets (m < 2^32 is required)
+//   adj   u32[m]    packed edge word dst | (w-1) << dbits      (when w_max-1 fits the high bits)
+//   adjw  uint2[m]  (dst, w) pairs                              (otherwise)
+//   big   u32[ceil(n/32)] bit v set iff outdeg(v) >= BIG_T (rows split into CHUNK-edge pieces)
+struct Adj {
+    uint32_t n = 0, m = 0;
+    DevBuf<uint32_t> ptr;
+    DevBuf<uint32_t> adj;
+    DevBuf<uint2> adjw;
+    DevBuf<uint32_t> big;
+};
+
+struct GraphView {
+    const uint32_t* ptr;
+    const uint32_t* adj;
+    const uint2* adjw;
+    const uint32_t* big;
+};
+
+inline GraphView view(const Adj& a) { return GraphView{a.ptr.get(), a.adj.get(), a.adjw.get(), a.big.get()}; }
+
+struct Core {
+    bool built = false;
+    int alg = 0;           // 1 = Algorithm 1 (specialized), 2 = Algorithm 2 (general)
+    int connectivity = 0;
+    Adj adj;               // CG(V, E_c) in the engine layout
+    DevBuf<uint8_t> flags; // E_c membership in G's CSR edge order
+    std::vector<uint32_t> hubs;
+    float build_ms = 0.f;
+};
+
+struct Workspace {
+    uint32_t n = 0;
+    DevBuf<uint32_t> bitmap;                // ceil(n/32) frontier bits
+    DevBuf<uint32_t> list;                  // n compacted frontier ids
+    DevBuf<uint2> big;                      // (vertex, first chunk) of high-degree frontier rows
+    DevBuf<unsigned long long> ctrl;        // grid barrier + per-iteration counters
+    DevBuf<unsigned long long> stats;       // per-query counters
+    DevBuf<uint32_t> err;                   // error flag
+    uint32_t big_cap = 0;
+    uint32_t stats_cap = 0;
+};
+
+struct Graph {
+    int device = 0;
+    uint32_t n = 0, m = 0, w_max = 0;
+    uint32_t dbits = 0;    // bits of the destination id in a packed edge word
+    bool packed = false;
+    int num_sms = 0;
+    Adj g;                 // CSR of G
+    Adj gr;                // CSR of G^R (= CSC of G)
+    DevBuf<uint32_t> reid; // CSC position -> CSR edge index
+    Core core[6];          // indexed by cg_kind (BFS uses the REACH slot: one general CG)
+    Workspace ws;
+};
+
+inline int core_slot(int kind) { return kind == CG_BFS ? CG_REACH : kind; }
+
+// graph_build.cu
+void build_graph(Graph& G, int64_t n, int64_t m, const uint32_t* src, const uint32_t* dst, const uint32_t* w,
+                 cudaStream_t s);
+void build_big_bitmap(Adj& a, cudaStream_t s);
+void export_adj(const Graph& G, const Adj& a, int64_t* ptr, uint32_t* idx, uint32_t* w, cudaStream_t s);
+
+// engine.cu
+struct QueryCall {
+    int kind;
+    GraphView full;        // G (or G^R for backward Identify queries)
+    GraphView core;        // CG (phase 1); ignored when two_phase == 0
+    int two_phase;
+    const uint32_t* srcs;  // device
+    int32_t n_src;
+    uint32_t* out;         // n_src * n
+    uint32_t* p1;          // nullable
+    bool want_stats;
+};
+void run_queries(Graph& G, const QueryCall& c, cudaStream_t s, std::vector<cg_stats>* stats);
+
+// core_graph.cu
+void build_core(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs, uint64_t seed, int alg,
+                int connectivity, cudaStream_t s);
+
+// gen.cu
+void rmat_generate(uint64_t n, uint32_t tA, uint32_t tAB, uint32_t tABC, uint32_t w_max, uint64_t seed, int permute,
+                   uint64_t e0, uint64_t count, uint32_t* src, uint32_t* dst, uint32_t* w, cudaStream_t s);
+
+}  // namespace cgb

@@ -1,0 +1,222 @@
+"""GPU parity: the CUDA path through the C ABI vs the CPU oracle, element by element.
+
+Bars: CSR/CSC, CG edge sets, hub ids and all integer-kind values are
+bit-exact; Viterbi values are bit-exact too (fallback bound 1e-6 relative, north_star).
+"""
+import numpy as np
+import pytest
+import torch
+
+import gen
+import oracle
+from gpu_util import assert_values_equal, both, gpu_graph, to_dev, to_np
+from helpers import KINDS, random_multigraph
+
+pytestmark = pytest.mark.gpu
+
+
+# ------------------------------------------------------------------ inputs
+def test_device_generator_matches_host():
+    from paper_conf_eurosys_0002a0a024_b200 import rmat_device
+    for n, m, seed, permute, wm in ((1 << 12, 50_000, 1, True, 64), (4_847_571, 200_000, 2, True, 23),
+                                   (1000, 30_000, 3, False, 7), (3, 100, 4, True, 1)):
+        hs, hd, hw = gen.rmat(n, m, w_max=wm, seed=seed, permute=permute)
+        ds, dd, dw = rmat_device(n, m, w_max=wm, seed=seed, permute=permute, device="cuda:0")
+        assert np.array_equal(to_np(ds), hs) and np.array_equal(to_np(dd), hd) and np.array_equal(to_np(dw), hw)
+
+
+# ------------------------------------------------------------------ a1, a2: CSR / CSC
+@pytest.mark.parametrize("seed", range(6))
+def test_csr_csc_bit_equal(seed):
+    rng = np.random.default_rng(seed)
+    n = int(rng.integers(1, 3000))
+    src, dst, w = random_multigraph(rng, n, int(rng.integers(0, 20000)), wset=tuple(range(1, 70)))
+    g, og = both(n, src, dst, w)
+    assert g.m == og.m
+    ptr, idx, ww = g.export()
+    assert np.array_equal(ptr.cpu().numpy(), og.ptr)
+    assert np.array_equal(to_np(idx), og.col) and np.array_equal(to_np(ww), og.wt)
+    ogr = oracle.transpose(og)
+    ptr, idx, ww = g.export(transpose=True)
+    assert np.array_equal(ptr.cpu().numpy(), ogr.ptr)
+    assert np.array_equal(to_np(idx), ogr.col) and np.array_equal(to_np(ww), ogr.wt)
+
+
+def test_csr_rmat16_and_wide_weights():
+    n, m = 1 << 16, 16 << 16
+    for wm in (64, 1 << 20):   # packed edge words, then the (dst, w) pair layout
+        src, dst, w = gen.rmat(n, m, w_max=wm, seed=1)
+        g, og = both(n, src, dst, w)
+        ptr, idx, ww = g.export()
+        assert np.array_equal(ptr.cpu().numpy(), og.ptr)
+        assert np.array_equal(to_np(idx), og.col) and np.array_equal(to_np(ww), og.wt)
+
+
+def test_graph_input_errors():
+    from paper_conf_eurosys_0002a0a024_b200 import CGInvalid
+    with pytest.raises(CGInvalid):
+        gpu_graph(4, np.array([0, 9]), np.array([1, 2]), np.array([1, 1]))
+    with pytest.raises(CGInvalid):
+        gpu_graph(4, np.array([0, 1]), np.array([1, 2]), np.array([1, 0]))
+
+
+# ------------------------------------------------------------------ a8-a13: queries
+def _check_queries(n, src, dst, w, sources, kinds=KINDS, modes=("full", "2phase"), K=8):
+    g, og = both(n, src, dst, w)
+    ogr = oracle.transpose(og)
+    for kind in kinds:
+        if "2phase" in modes:
+            g.build(kind, K=min(K, n))
+        for mode in modes:
+            out = to_np(g.query(kind, to_dev(sources), mode=mode))
+            for i, s in enumerate(sources):
+                assert_values_equal(out[i], oracle.query(kind, og, int(s)), kind, f"{kind}/{mode}/s={s}")
+    g.close()
+    return og, ogr
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_queries_small_random(seed):
+    rng = np.random.default_rng(seed)
+    n = int(rng.integers(1, 200))
+    src, dst, w = random_multigraph(rng, n, int(rng.integers(0, 6 * n + 1)))
+    _check_queries(n, src, dst, w, np.arange(n, dtype=np.uint32))
+
+
+def test_queries_rmat16_config1():
+    """configs[0]: RMAT scale-16 ef16, w 1..64 — vertex 0 (the config's query) + 64 sampled sources."""
+    c = gen.CONFIGS["c1"]
+    src, dst, w = c.edges()
+    sources = np.concatenate([[0], gen.sample_sources(c.n, src, dst, 64, seed=42)]).astype(np.uint32)
+    _check_queries(c.n, src, dst, w, sources, K=20)
+
+
+def test_edge_cases():
+    # n = 1, no edges
+    _check_queries(1, np.zeros(0, np.uint32), np.zeros(0, np.uint32), np.zeros(0, np.uint32), np.array([0], np.uint32),
+                   K=1)
+    # isolated source and a source with outdeg 0 in a two-component graph with self-loops, duplicates
+    src = np.array([0, 0, 1, 2, 2, 4, 5, 5, 6], np.uint32)
+    dst = np.array([1, 1, 2, 0, 2, 5, 6, 6, 4], np.uint32)
+    w = np.array([3, 2, 64, 1, 5, 1, 7, 3, 2], np.uint32)
+    _check_queries(8, src, dst, w, np.arange(8, dtype=np.uint32), K=2)
+
+
+def test_long_chain_loop_control():
+    n = 100_000
+    src = np.arange(n - 1, dtype=np.uint32)
+    dst = src + 1
+    w = (src % 7 + 1).astype(np.uint32)
+    _check_queries(n, src, dst, w, np.array([0, n // 2], np.uint32), kinds=("sssp", "bfs", "viterbi", "reach"),
+                   modes=("full",))
+
+
+def test_star_hub_chunks():
+    """A hub with 10^6 out-edges exercises the multi-CTA chunk tier (rows >= kBigThreshold)."""
+    leaves = 1_000_000
+    n = leaves + 2
+    src = np.concatenate([np.zeros(leaves, np.uint32), np.arange(1, 2001, dtype=np.uint32)])
+    dst = np.concatenate([np.arange(1, leaves + 1, dtype=np.uint32), np.full(2000, n - 1, np.uint32)])
+    rng = np.random.default_rng(3)
+    w = rng.integers(1, 65, size=src.size).astype(np.uint32)
+    _check_queries(n, src, dst, w, np.array([0, 5], np.uint32), kinds=("sssp", "sswp", "reach"), K=2)
+
+
+def test_viterbi_powers_of_two_exact():
+    n, m = 1 << 12, 16 << 12
+    src, dst, _ = gen.rmat(n, m, seed=6)
+    rng = np.random.default_rng(6)
+    w = (1 << rng.integers(1, 7, size=m)).astype(np.uint32)
+    _check_queries(n, src, dst, w, np.arange(0, n, 97, dtype=np.uint32), kinds=("viterbi",))
+
+
+# ------------------------------------------------------------------ a3-a7: Core Graph
+@pytest.mark.parametrize("kind", KINDS)
+def test_core_graph_edge_set_and_hubs(kind):
+    n, m = 1 << 14, 16 << 14
+    src, dst, w = gen.rmat(n, m, w_max=15, seed=11)
+    g, og = both(n, src, dst, w)
+    ogr = oracle.transpose(og)
+    info = g.build(kind, K=20)
+    hubs = oracle.hubs_topdeg(og, ogr, 20)
+    assert info["hubs"] == [int(h) for h in hubs]
+    exp = oracle.cg_for_kind(kind, og, ogr, hubs)
+    got = g.core_flags(kind).cpu().numpy()
+    assert got.size == exp.size
+    bad = np.nonzero(got != exp)[0]
+    assert bad.size == 0, f"{kind}: {bad.size} CG edges differ"
+    assert info["m_cg"] == int(exp.sum())
+
+
+@pytest.mark.parametrize("kind", KINDS)
+def test_phase1_values_and_precision(kind):
+    """p1 (the phase-1 fixpoint on CG) and impacted / reached / precise counts are unique: equal
+    to the oracle's Alg 3."""
+    n, m = 1 << 13, 16 << 13
+    src, dst, w = gen.rmat(n, m, w_max=31, seed=5)
+    g, og = both(n, src, dst, w)
+    ogr = oracle.transpose(og)
+    g.build(kind, K=20)
+    cg = oracle.subgraph(og, oracle.cg_for_kind(kind, og, ogr, oracle.hubs_topdeg(og, ogr, 20)))
+    sources = gen.sample_sources(n, src, dst, 16, seed=9)
+    out, p1, stats = g.query(kind, to_dev(sources), mode="2phase", p1=True, stats=True)
+    out, p1 = to_np(out), to_np(p1)
+    for i, s in enumerate(sources):
+        val, op1, st = oracle.two_phase(kind, og, cg, int(s))
+        assert_values_equal(out[i], val, kind, f"final s={s}")
+        assert_values_equal(p1[i], op1, kind, f"p1 s={s}")
+        assert stats[i]["reached"] == st["reached"]
+        assert stats[i]["precise_p1"] == st["precise_p1"]
+        assert stats[i]["impacted"] == st["impacted"]
+
+
+def test_hub_policies_and_errors():
+    from paper_conf_eurosys_0002a0a024_b200 import CGInvalid, CGNoCoreGraph
+    n, m = 1 << 12, 8 << 12
+    src, dst, w = gen.rmat(n, m, seed=2)
+    g, og = both(n, src, dst, w)
+    with pytest.raises(CGNoCoreGraph):
+        g.query("sssp", to_dev(np.array([1], np.uint32)), mode="2phase")
+    with pytest.raises(CGInvalid):
+        g.build("sssp", K=0)
+    with pytest.raises(CGInvalid):
+        g.build("sssp", hubs=[n + 5])
+    with pytest.raises(CGInvalid):
+        g.query("sssp", to_dev(np.array([n], np.uint32)), mode="full", stats=True)
+    info = g.build("sssp", hubs=[3, 17, 99])
+    assert info["hubs"] == [3, 17, 99]
+    ogr = oracle.transpose(og)
+    exp = oracle.cg_alg1("sssp", og, ogr, np.array([3, 17, 99], np.uint32))
+    got = g.core_flags("sssp").cpu().numpy()
+    assert np.array_equal(got, exp)
+    info = g.build("sswp", K=10, policy="sampled", seed=123)
+    assert len(set(info["hubs"])) == 10
+    s = gen.sample_sources(n, src, dst, 8, seed=1)
+    out = to_np(g.query("sswp", to_dev(s), mode="2phase"))
+    for i, x in enumerate(s):
+        assert_values_equal(out[i], oracle.query("sswp", og, int(x)), "sswp")
+
+
+def test_query_host_end_to_end():
+    n, m = 1 << 14, 16 << 14
+    src, dst, w = gen.rmat(n, m, seed=4)
+    g, og = both(n, src, dst, w)
+    g.build("ssnp", K=20)
+    s = gen.sample_sources(n, src, dst, 7, seed=3)
+    out = g.query_host("ssnp", torch.from_numpy(s.astype(np.int64)), mode="2phase", batch=3)
+    got = out.view(torch.int32).numpy().view(np.uint32)
+    for i, x in enumerate(s):
+        assert_values_equal(got[i], oracle.query("ssnp", og, int(x)), "ssnp")
+
+
+def test_alg_options_match_oracle():
+    """Alg 1 for REACH/BFS and Alg 2 with connectivity (the options of readings Q11/Q12)."""
+    n, m = 1 << 12, 12 << 12
+    src, dst, w = gen.rmat(n, m, seed=8)
+    g, og = both(n, src, dst, w)
+    ogr = oracle.transpose(og)
+    hubs = oracle.hubs_topdeg(og, ogr, 10)
+    g.build("bfs", K=10, alg="specialized")
+    assert np.array_equal(g.core_flags("bfs").cpu().numpy(), oracle.cg_alg1("bfs", og, ogr, hubs))
+    g.build("reach", K=10, alg="general", connectivity=True)
+    assert np.array_equal(g.core_flags("reach").cpu().numpy(), oracle.cg_alg2(og, ogr, hubs, connectivity=True))
