@@ -72,7 +72,7 @@ typedef struct cg_graph_s* cg_graph; /* opaque: owns G (CSR), G^R (CSC) and the 
 typedef struct {
     int64_t iters_p1, iters_p2;      /* BSP iterations of phase 1 (CG) and phase 2 (G or FULL) */
     int64_t edges_p1, edges_p2;      /* edges scanned by Process (Alg 3 l.24) */
-    int64_t updates_p1, updates_p2;  /* successful CASMIN/CASMAX EdgeFunction updates (l.26) */
+    int64_t updates_p1, updates_p2;  /* EdgeFunction calls (l.26): CASMIN/CASMAX atomics issued when Needed (Fig 5 ATOMIC) */
     int64_t frontier_p1, frontier_p2;/* sum over iterations of |Active| */
     int64_t impacted;                /* |Active| at the start of phase 2 (Alg 3 l.15, reading Q4) */
     int64_t reached;                 /* |{v != s : Val(v) != InitVal}| after the query */

@@ -98,11 +98,14 @@ def lib(build: bool = True) -> ctypes.CDLL:
     """Load (building first if stale) the CUDA library.  Raises if it cannot be produced."""
     global _lib
     if _lib is None:
-        if build:
-            _build.build()
-        if not os.path.exists(_build.LIB):
-            raise ImportError(f"CUDA library {_build.LIB} is missing (no CPU fallback exists)")
-        L = ctypes.CDLL(_build.LIB)
+        path = os.environ.get("CGB_LIB")  # an experiment variant built by _build.build(out=...)
+        if not path:
+            if build:
+                _build.build()
+            path = _build.LIB
+        if not os.path.exists(path):
+            raise ImportError(f"CUDA library {path} is missing (no CPU fallback exists)")
+        L = ctypes.CDLL(path)
         for name, (res, args) in _SIGS.items():
             f = getattr(L, name)
             f.restype = res

@@ -229,8 +229,8 @@ cg_status cg_query_ex(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_s
             CGB_CHECK(!hb, CG_EINVAL, "source id >= n");
         }
         const bool two = mode == CG_MODE_2PHASE;
-        QueryCall c{(int)kind, view(G.g), two ? view(G.core[core_slot(kind)].adj) : view(G.g), two ? 1 : 0, src,
-                    n_src, (uint32_t*)out, two ? (uint32_t*)p1_out : nullptr, stats != nullptr};
+        QueryCall c{(int)kind, &G.g, two ? &G.core[core_slot(kind)].adj : &G.g, two ? 1 : 0, src, n_src,
+                    (uint32_t*)out, two ? (uint32_t*)p1_out : nullptr, stats != nullptr};
         std::vector<cg_stats> st;
         run_queries(G, c, S(stream), stats ? &st : nullptr);
         if (stats) std::memcpy(stats, st.data(), sizeof(cg_stats) * (size_t)n_src);
@@ -276,8 +276,8 @@ cg_status cg_query_host(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n
             const int32_t nq = (n_src - q0) < batch ? (n_src - q0) : batch;
             const int k = b & 1;
             if (b >= 2) CGB_CUDA(cudaStreamWaitEvent(s, drained[k], 0));
-            QueryCall c{(int)kind, view(G.g), two ? view(G.core[core_slot(kind)].adj) : view(G.g), two ? 1 : 0,
-                        dsrc.get() + q0, nq, slot[k].get(), nullptr, false};
+            QueryCall c{(int)kind, &G.g, two ? &G.core[core_slot(kind)].adj : &G.g, two ? 1 : 0, dsrc.get() + q0,
+                        nq, slot[k].get(), nullptr, false};
             run_queries(G, c, s, nullptr);
             CGB_CUDA(cudaEventRecord(done[k], s));
             CGB_CUDA(cudaStreamWaitEvent(cp, done[k], 0));

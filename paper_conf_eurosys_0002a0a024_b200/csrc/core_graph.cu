@@ -312,9 +312,9 @@ void alg1(Graph& G, int kind, const std::vector<uint32_t>& hubs, uint8_t* flags,
     DevBuf<uint32_t> vf((size_t)group * G.n, s), vb((size_t)group * G.n, s);
     for (int k0 = 0; k0 < K; k0 += group) {
         const int nh = (K - k0) < group ? (K - k0) : group;
-        QueryCall f{kind, view(G.g), view(G.g), 0, hsrc.get() + k0, nh, vf.get(), nullptr, false};
+        QueryCall f{kind, &G.g, &G.g, 0, hsrc.get() + k0, nh, vf.get(), nullptr, false};
         run_queries(G, f, s, nullptr);                   // Alg 1 l.4: Identify(G, forward)
-        QueryCall b{kind, view(G.gr), view(G.gr), 0, hsrc.get() + k0, nh, vb.get(), nullptr, false};
+        QueryCall b{kind, &G.gr, &G.gr, 0, hsrc.get() + k0, nh, vb.get(), nullptr, false};
         run_queries(G, b, s, nullptr);                   // Alg 1 l.5: Identify(G^R, backward)
         switch (kind) {
         case CG_SSSP: mark_group<CG_SSSP>(G, nh, vf.get(), vb.get(), flags, s); break;
@@ -416,10 +416,9 @@ void build_core(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs_
     C.adj.m = mcg;
     C.adj.adj.reset();
     C.adj.adjw.reset();
-    if (G.packed) C.adj.adj.alloc(mcg ? mcg : 1, s); else C.adj.adjw.alloc(mcg ? mcg : 1, s);
+    if (G.packed) C.adj.adj.alloc(adj_alloc_elems(mcg, 4), s); else C.adj.adjw.alloc(adj_alloc_elems(mcg, 8), s);
     CGB_LAUNCH(k_scatter_core, grid_rows(G.n), TB, 0, s, G.n, G.g.ptr.get(), C.flags.get(), C.adj.ptr.get(),
                G.g.adj.get(), G.g.adjw.get(), C.adj.adj.get(), C.adj.adjw.get());
-    build_big_bitmap(C.adj, s);
     CGB_CUDA(cudaEventRecord(e1, s));
     CGB_CUDA(cudaEventSynchronize(e1));
     float ms = 0.f;

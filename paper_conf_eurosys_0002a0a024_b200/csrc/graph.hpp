@@ -7,32 +7,29 @@
 
 namespace cgb {
 
-// Rows with at least kBigThreshold out-edges are split into kChunk-edge pieces that all
-// warps of the grid share (the "CTA-per-high-degree" tier, generalised to multi-CTA).
-constexpr uint32_t kBigThreshold = 2048;
-constexpr uint32_t kChunk = 512;
+// Edge arrays are over-allocated by this many bytes so that vectorised / bulk edge reads may
+// run past the last edge without leaving the allocation.
+constexpr size_t kAdjPadBytes = 4096;
+inline size_t adj_alloc_elems(size_t m, size_t elem_bytes) { return m + kAdjPadBytes / elem_bytes; }
 
 // Out-edge structure in the engine's HBM layout:
 //   ptr   u32[n+1]  row offsets (m < 2^32 is required)
 //   adj   u32[m]    packed edge word dst | (w-1) << dbits      (when w_max-1 fits the high bits)
 //   adjw  uint2[m]  (dst, w) pairs                              (otherwise)
-//   big   u32[ceil(n/32)] bit v set iff outdeg(v) >= BIG_T (rows split into CHUNK-edge pieces)
 struct Adj {
     uint32_t n = 0, m = 0;
     DevBuf<uint32_t> ptr;
     DevBuf<uint32_t> adj;
     DevBuf<uint2> adjw;
-    DevBuf<uint32_t> big;
 };
 
 struct GraphView {
     const uint32_t* ptr;
     const uint32_t* adj;
     const uint2* adjw;
-    const uint32_t* big;
 };
 
-inline GraphView view(const Adj& a) { return GraphView{a.ptr.get(), a.adj.get(), a.adjw.get(), a.big.get()}; }
+inline GraphView view(const Adj& a) { return GraphView{a.ptr.get(), a.adj.get(), a.adjw.get()}; }
 
 struct Core {
     bool built = false;
@@ -47,12 +44,11 @@ struct Core {
 struct Workspace {
     uint32_t n = 0;
     DevBuf<uint32_t> bitmap;                // ceil(n/32) frontier bits
-    DevBuf<uint32_t> list;                  // n compacted frontier ids
-    DevBuf<uint2> big;                      // (vertex, first chunk) of high-degree frontier rows
+    DevBuf<uint32_t> lv;                    // n compacted frontier ids
+    DevBuf<uint32_t> lo;                    // n exclusive edge offsets of the frontier rows
     DevBuf<unsigned long long> ctrl;        // grid barrier + per-iteration counters
     DevBuf<unsigned long long> stats;       // per-query counters
     DevBuf<uint32_t> err;                   // error flag
-    uint32_t big_cap = 0;
     uint32_t stats_cap = 0;
 };
 
@@ -74,14 +70,13 @@ inline int core_slot(int kind) { return kind == CG_BFS ? CG_REACH : kind; }
 // graph_build.cu
 void build_graph(Graph& G, int64_t n, int64_t m, const uint32_t* src, const uint32_t* dst, const uint32_t* w,
                  cudaStream_t s);
-void build_big_bitmap(Adj& a, cudaStream_t s);
 void export_adj(const Graph& G, const Adj& a, int64_t* ptr, uint32_t* idx, uint32_t* w, cudaStream_t s);
 
 // engine.cu
 struct QueryCall {
     int kind;
-    GraphView full;        // G (or G^R for backward Identify queries)
-    GraphView core;        // CG (phase 1); ignored when two_phase == 0
+    Adj* full_adj;         // G (or G^R for backward Identify queries)
+    Adj* core_adj;         // CG (phase 1); ignored when two_phase == 0
     int two_phase;
     const uint32_t* srcs;  // device
     int32_t n_src;

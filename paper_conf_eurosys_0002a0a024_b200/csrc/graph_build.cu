@@ -116,18 +116,6 @@ __global__ void k_split_keys(uint32_t m, const unsigned long long* __restrict__ 
     }
 }
 
-__global__ void k_big_bitmap(uint32_t n, const uint32_t* __restrict__ ptr, uint32_t thresh, uint32_t* __restrict__ big) {
-    uint32_t words = (n + 31) / 32;
-    for (uint64_t wi = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; wi < words; wi += (uint64_t)gridDim.x * blockDim.x) {
-        uint32_t bits = 0;
-        for (uint32_t j = 0; j < 32; ++j) {
-            uint64_t v = wi * 32 + j;
-            if (v < n && ptr[v + 1] - ptr[v] >= thresh) bits |= 1u << j;
-        }
-        big[wi] = bits;
-    }
-}
-
 __global__ void k_export(uint32_t n, uint32_t m, uint32_t dbits, const uint32_t* __restrict__ ptr32,
                          const uint32_t* __restrict__ adj, const uint2* __restrict__ adjw, int64_t* __restrict__ ptr,
                          uint32_t* __restrict__ idx, uint32_t* __restrict__ w) {
@@ -163,12 +151,6 @@ void exclusive_sum(const uint32_t* in, uint32_t* out, uint64_t m, cudaStream_t s
 }
 
 }  // namespace
-
-void build_big_bitmap(Adj& a, cudaStream_t s) {
-    uint32_t words = (a.n + 31) / 32;
-    a.big.alloc(words ? words : 1, s);
-    CGB_LAUNCH(k_big_bitmap, grid_for(words), TB, 0, s, a.n, a.ptr.get(), kBigThreshold, a.big.get());
-}
 
 void build_graph(Graph& G, int64_t n64, int64_t m64, const uint32_t* src, const uint32_t* dst, const uint32_t* w,
                  cudaStream_t s) {
@@ -229,16 +211,15 @@ void build_graph(Graph& G, int64_t n64, int64_t m64, const uint32_t* src, const 
     // 4. CSR of G
     G.g.ptr.alloc(n + 1, s);
     CGB_LAUNCH(k_row_ptr, grid_for((uint64_t)mc + 1), TB, 0, s, mc, n, csrc.get(), G.g.ptr.get());
-    if (G.packed) G.g.adj.alloc(mc ? mc : 1, s); else G.g.adjw.alloc(mc ? mc : 1, s);
+    if (G.packed) G.g.adj.alloc(adj_alloc_elems(mc, 4), s); else G.g.adjw.alloc(adj_alloc_elems(mc, 8), s);
     if (mc)
         CGB_LAUNCH(k_pack, grid_for(mc), TB, 0, s, mc, G.dbits, (int)G.packed, cdst.get(), cw.get(),
                    (const uint32_t*)nullptr, G.g.adj.get(), G.g.adjw.get());
-    build_big_bitmap(G.g, s);
 
     // 5. G^R: sort (dst, src) with the CSR edge index as value
     G.gr.ptr.alloc(n + 1, s);
     G.reid.alloc(mc ? mc : 1, s);
-    if (G.packed) G.gr.adj.alloc(mc ? mc : 1, s); else G.gr.adjw.alloc(mc ? mc : 1, s);
+    if (G.packed) G.gr.adj.alloc(adj_alloc_elems(mc, 4), s); else G.gr.adjw.alloc(adj_alloc_elems(mc, 8), s);
     {
         DevBuf<uint32_t> rsrc(mc ? mc : 1, s), rrow(mc ? mc : 1, s);
         if (mc) {
@@ -253,7 +234,6 @@ void build_graph(Graph& G, int64_t n64, int64_t m64, const uint32_t* src, const 
             CGB_LAUNCH(k_pack, grid_for(mc), TB, 0, s, mc, G.dbits, (int)G.packed, rrow.get(), cw.get(),
                        G.reid.get(), G.gr.adj.get(), G.gr.adjw.get());
     }
-    build_big_bitmap(G.gr, s);
     CGB_CUDA(cudaStreamSynchronize(s));
 }
 

@@ -220,3 +220,21 @@ def test_alg_options_match_oracle():
     assert np.array_equal(g.core_flags("bfs").cpu().numpy(), oracle.cg_alg1("bfs", og, ogr, hubs))
     g.build("reach", K=10, alg="general", connectivity=True)
     assert np.array_equal(g.core_flags("reach").cpu().numpy(), oracle.cg_alg2(og, ogr, hubs, connectivity=True))
+
+
+@pytest.mark.parametrize("dense_div", ["0", "8", "4294967295"])
+def test_dense_and_sparse_iterations(dense_div, monkeypatch):
+    """Force every iteration sparse (list + balanced split), the default mix, or every
+    iteration dense (TMA-streamed edge slices): all must give the oracle's values.  A graph
+    large enough for multi-chunk slices, skipped inactive hub rows and many warps per row."""
+    monkeypatch.setenv("CG_DENSE_DIV", dense_div)
+    n, m = 1 << 18, 16 << 18
+    src, dst, w = gen.rmat(n, m, w_max=19, seed=13)
+    g, og = both(n, src, dst, w)
+    sources = np.concatenate([[0], gen.sample_sources(n, src, dst, 5, seed=2)]).astype(np.uint32)
+    for kind in ("sssp", "viterbi", "bfs", "sswp"):
+        g.build(kind, K=20)
+        for mode in ("full", "2phase"):
+            out = to_np(g.query(kind, to_dev(sources), mode=mode))
+            for i, s in enumerate(sources):
+                assert_values_equal(out[i], oracle.query(kind, og, int(s)), kind, f"{kind}/{mode}/div={dense_div}/s={s}")
