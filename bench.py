@@ -130,9 +130,6 @@ def dist_setup():
     return rank, ws, local
 
 
-def shard_seed(base: int, rank: int) -> int:
-    """Each rank draws its own sources: weak scaling over independent vertex queries."""
-    return base + 7919 * rank
 
 
 def host_edges(cfg):
@@ -140,9 +137,14 @@ def host_edges(cfg):
     return gen.rmat(cfg.n, cfg.m, cfg.abcd, cfg.w_max, cfg.seed)
 
 
-def sources_for(cfg, src_h, dst_h, kind_idx, count, rank):
+def sources_for(cfg, src_h, dst_h, kind_idx, count, rank, world=1):
+    """Rank's contiguous shard of the kind's global seeded source list (count per rank: weak
+    scaling over independent vertex queries)."""
     import gen
-    return gen.sample_sources(cfg.n, src_h, dst_h, count, seed=shard_seed(1000 + 17 * kind_idx, rank))
+    from paper_conf_eurosys_0002a0a024_b200 import multi
+    allsrc = gen.sample_sources(cfg.n, src_h, dst_h, count * world, seed=1000 + 17 * kind_idx)
+    a, b = multi.shard(len(allsrc), rank, world)
+    return allsrc[a:b]
 
 
 # ---------------------------------------------------------------------------- CPU oracle arm
@@ -203,7 +205,7 @@ def main():
     import torch
 
     import gen
-    from paper_conf_eurosys_0002a0a024_b200 import Graph, kernel_launches, rmat_device
+    from paper_conf_eurosys_0002a0a024_b200 import Graph, kernel_launches, multi, rmat_device
 
     rank, ws, local = dist_setup()
     dev = torch.device("cuda", local)
@@ -232,7 +234,7 @@ def main():
     ptr, _, _ = g.export()
     outdeg = (ptr[1:] - ptr[:-1]).to(torch.int64)
     del ptr
-    srcs = {k: torch.from_numpy(sources_for(cfg, src_h, dst_h, KINDS.index(k), B, rank).astype(np.int64))
+    srcs = {k: torch.from_numpy(sources_for(cfg, src_h, dst_h, KINDS.index(k), B, rank, ws).astype(np.int64))
             .to(torch.uint32).to(dev) for k in kinds}
     nbuf = 2 if gather else 1
     outs = [{k: torch.empty((B, cfg.n), dtype=torch.uint32, device=dev) for k in kinds} for _ in range(nbuf)]
@@ -257,9 +259,9 @@ def main():
             if events is not None:
                 events[k][1].record(stream)
         if gather and works is not None:
-            import torch.distributed as dist
             for k in kinds:
-                works.append(dist.gather(o[k], gathered[k] if rank == 0 else None, dst=0, async_op=True))
+                _, wk = multi.gather_rows(o[k], rank, ws, gathered[k] if rank == 0 else None, async_op=True)
+                works.append(wk)
 
     def timed(mode, steps, with_events=True):
         for i in range(args.warmup):
@@ -279,12 +281,7 @@ def main():
         end.record(stream)
         barrier()
         launches = kernel_launches() - l0
-        ms = start.elapsed_time(end)
-        if ws > 1:
-            import torch.distributed as dist
-            t = torch.tensor([ms], device=dev, dtype=torch.float64)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            ms = float(t.item())
+        ms = multi.max_over_ranks(start.elapsed_time(end), dev)
         per_kind_ms = {k: [e[k][0].elapsed_time(e[k][1]) for e in evs] for k in kinds} if with_events else None
         return ms, per_kind_ms, launches
 
@@ -378,12 +375,7 @@ def main():
             for k in kinds:
                 g.query_host(k, hsrc[k], mode="2phase", out=hout[k])
         barrier()
-        el = time.perf_counter() - t0
-        if ws > 1:
-            import torch.distributed as dist
-            t = _t.tensor([el], device=dev, dtype=_t.float64)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            el = float(t.item())
+        el = multi.max_over_ranks(time.perf_counter() - t0, dev)
         e2e = {"value": ws * q_step * steps_e2e / el, "unit": "queries/s", "h2d_bytes_per_step": 4 * q_step,
                "d2h_bytes_per_step": 4 * q_step * cfg.n, "api": "cg_query_host (pinned host buffers)",
                "steps": steps_e2e}

@@ -5,6 +5,7 @@ Viterbi, BFS and REACH, behind the C ABI in include/cg.h.
 The CUDA library (csrc/ -> libcoregraph_b200.so) is the only compute path; there is no CPU
 fallback.  ``Graph`` marshals tensors to the ABI.
 """
+from . import multi  # noqa: F401
 from .graph import CG_ALGS, HUB_POLICIES, KINDS, MODES, Graph, kernel_launches, kind_id, rmat_device  # noqa: F401
 from ._lib import CGError, CGInvalid, CGNoCoreGraph, CGOverflow  # noqa: F401
 

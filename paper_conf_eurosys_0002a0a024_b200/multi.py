@@ -1,0 +1,42 @@
+"""Multi-GPU plumbing for batches of independent vertex queries.
+
+Vertex queries are independent: the source list is split into contiguous shards,
+one per rank (each GPU holds a full replica of G and its Core Graphs), and the only exchange
+is gathering the value rows to rank 0.  torch.distributed provides the transport (NCCL over
+NVLink / NVSwitch on GPUs, gloo in the CPU tests); nothing here computes.
+"""
+from __future__ import annotations
+
+import torch
+import torch.distributed as dist
+
+
+def shard(n_total: int, rank: int, world: int) -> tuple[int, int]:
+    """[start, stop) of rank's contiguous shard; shard sizes differ by at most one."""
+    if world <= 0 or not 0 <= rank < world:
+        raise ValueError("bad rank / world size")
+    base, extra = divmod(n_total, world)
+    start = rank * base + min(rank, extra)
+    return start, start + base + (1 if rank < extra else 0)
+
+
+def gather_rows(values: torch.Tensor, rank: int, world: int, root_buffers=None, async_op: bool = False):
+    """Gather every rank's [rows, n] value block to rank 0 (equal row counts per rank).
+
+    root_buffers: on rank 0, a list of `world` tensors shaped like `values` (allocated here if
+    None).  Returns (buffers on rank 0 / None elsewhere, work handle or None)."""
+    if world == 1:
+        return [values], None
+    if rank == 0 and root_buffers is None:
+        root_buffers = [torch.empty_like(values) for _ in range(world)]
+    work = dist.gather(values, root_buffers if rank == 0 else None, dst=0, async_op=async_op)
+    return (root_buffers if rank == 0 else None), work
+
+
+def max_over_ranks(x: float, device=None) -> float:
+    """Max of a host scalar over all ranks (timing is reported as the slowest rank)."""
+    if not dist.is_available() or not dist.is_initialized() or dist.get_world_size() == 1:
+        return x
+    t = torch.tensor([x], dtype=torch.float64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())

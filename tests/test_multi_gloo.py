@@ -1,0 +1,75 @@
+"""World-size-2 gloo test of the multi-GPU host logic (sharding + gather to rank 0).
+
+Each rank evaluates its shard of the sources (with the CPU oracle standing in for a GPU — the
+CUDA path is exercised by the -m gpu tests) and the values are gathered to rank 0 with the same
+`paper_conf_eurosys_0002a0a024_b200.multi` functions bench.py uses; rank 0 must hold exactly
+the single-process result."""
+import os
+import socket
+import sys
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def _worker(rank, world, port, out_path):
+    sys.path.insert(0, ROOT)
+    import gen
+    import oracle
+    from paper_conf_eurosys_0002a0a024_b200 import multi
+
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    n = 1 << 10
+    src, dst, w = gen.rmat(n, 8 * n, seed=3)
+    g = oracle.canonical_csr(n, src, dst, w)
+    sources = gen.sample_sources(n, src, dst, 2 * world, seed=5)
+    a, b = multi.shard(len(sources), rank, world)
+    mine = torch.from_numpy(oracle.query_batch("sssp", g, sources[a:b]).view(np.int32))
+    bufs, work = multi.gather_rows(mine, rank, world, async_op=True)
+    work.wait()
+    t = multi.max_over_ranks(float(rank))
+    if rank == 0:
+        full = torch.cat(bufs).numpy().view(np.uint32)
+        np.save(out_path, full)
+        assert t == world - 1
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_shard_sizes():
+    from paper_conf_eurosys_0002a0a024_b200 import multi
+    for n in (0, 1, 7, 64, 129):
+        for world in (1, 2, 3, 8):
+            parts = [multi.shard(n, r, world) for r in range(world)]
+            assert parts[0][0] == 0 and parts[-1][1] == n
+            assert all(parts[i][1] == parts[i + 1][0] for i in range(world - 1))
+            sizes = [b - a for a, b in parts]
+            assert max(sizes) - min(sizes) <= 1
+    with pytest.raises(ValueError):
+        multi.shard(4, 2, 2)
+
+
+def test_gather_world2(tmp_path):
+    import gen
+    import oracle
+    out = str(tmp_path / "full.npy")
+    mp.spawn(_worker, args=(2, _free_port(), out), nprocs=2, join=True)
+    full = np.load(out)
+    n = 1 << 10
+    src, dst, w = gen.rmat(n, 8 * n, seed=3)
+    g = oracle.canonical_csr(n, src, dst, w)
+    sources = gen.sample_sources(n, src, dst, 4, seed=5)
+    assert np.array_equal(full, oracle.query_batch("sssp", g, sources))
