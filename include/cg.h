@@ -68,7 +68,10 @@ typedef struct cg_graph_s* cg_graph; /* opaque: owns G (CSR), G^R (CSC) and the 
 
 /* Per-query counters (SURVEY §5 tracing; Table 5 / Fig 5 analogs).  Edge and update
  * counts of the asynchronous GPU relaxation are NOT unique (they depend on timing);
- * impacted / reached / precise_p1 ARE unique. */
+ * impacted / reached / precise_p1 ARE unique.  When queries run batched (several sources per
+ * pass, the default for n_src >= 2), iterations and frontier sizes are those of the batch's
+ * union frontier and edges / updates are the batch's (edge, query) totals split evenly over
+ * its queries. */
 typedef struct {
     int64_t iters_p1, iters_p2;      /* BSP iterations of phase 1 (CG) and phase 2 (G or FULL) */
     int64_t edges_p1, edges_p2;      /* edges scanned by Process (Alg 3 l.24) */

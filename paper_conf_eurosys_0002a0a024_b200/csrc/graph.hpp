@@ -52,6 +52,16 @@ struct Workspace {
     uint32_t stats_cap = 0;
 };
 
+struct BatchSpace {         // engine_batch.cu workspace (B queries per pass)
+    uint32_t n = 0, B = 0;
+    DevBuf<uint32_t> V;         // [n][B] values
+    DevBuf<uint32_t> M;         // [n] active-query masks
+    DevBuf<uint32_t> bitmap;    // union frontier
+    DevBuf<uint32_t> lv, lo, lm;
+    DevBuf<unsigned long long> ctrl;
+    DevBuf<uint32_t> err;
+};
+
 struct Graph {
     int device = 0;
     uint32_t n = 0, m = 0, w_max = 0;
@@ -63,6 +73,7 @@ struct Graph {
     DevBuf<uint32_t> reid; // CSC position -> CSR edge index
     Core core[6];          // indexed by cg_kind (BFS uses the REACH slot: one general CG)
     Workspace ws;
+    BatchSpace bs;
 };
 
 inline int core_slot(int kind) { return kind == CG_BFS ? CG_REACH : kind; }
@@ -85,6 +96,10 @@ struct QueryCall {
     bool want_stats;
 };
 void run_queries(Graph& G, const QueryCall& c, cudaStream_t s, std::vector<cg_stats>* stats);
+
+// engine_batch.cu
+int batch_width();  // B of the batched engine (CG_BATCH env: 8 / 16 / 32; anything else disables it)
+void run_queries_batched(Graph& G, const QueryCall& c, int B, cudaStream_t s, std::vector<cg_stats>* stats);
 
 // core_graph.cu
 void build_core(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs, uint64_t seed, int alg,

@@ -238,3 +238,30 @@ def test_dense_and_sparse_iterations(dense_div, monkeypatch):
             out = to_np(g.query(kind, to_dev(sources), mode=mode))
             for i, s in enumerate(sources):
                 assert_values_equal(out[i], oracle.query(kind, og, int(s)), kind, f"{kind}/{mode}/div={dense_div}/s={s}")
+
+
+@pytest.mark.parametrize("batch", ["0", "8", "16", "32"])
+def test_single_and_batched_engines(batch, monkeypatch):
+    """CG_BATCH=0 runs every source through the single-query engine; 8/16/32 run B sources per
+    pass (NEXT-2, values laid out [n][B]).  A ragged tail (13 sources), all kinds, both modes,
+    phase-1 values and the unique per-query counts must match the oracle."""
+    monkeypatch.setenv("CG_BATCH", batch)
+    n, m = 1 << 14, 16 << 14
+    src, dst, w = gen.rmat(n, m, w_max=27, seed=21)
+    g, og = both(n, src, dst, w)
+    ogr = oracle.transpose(og)
+    hubs = oracle.hubs_topdeg(og, ogr, 20)
+    sources = np.concatenate([[0, 0], gen.sample_sources(n, src, dst, 11, seed=4)]).astype(np.uint32)
+    for kind in KINDS:
+        g.build(kind, K=20)
+        cg = oracle.subgraph(og, oracle.cg_for_kind(kind, og, ogr, hubs))
+        out, p1, st = g.query(kind, to_dev(sources), mode="2phase", p1=True, stats=True)
+        out, p1 = to_np(out), to_np(p1)
+        full = to_np(g.query(kind, to_dev(sources), mode="full"))
+        for i, s in enumerate(sources):
+            val, op1, ost = oracle.two_phase(kind, og, cg, int(s))
+            assert_values_equal(out[i], val, kind, f"B={batch} {kind} 2phase s={s}")
+            assert_values_equal(full[i], val, kind, f"B={batch} {kind} full s={s}")
+            assert_values_equal(p1[i], op1, kind, f"B={batch} {kind} p1 s={s}")
+            assert (st[i]["reached"], st[i]["precise_p1"], st[i]["impacted"]) == \
+                (ost["reached"], ost["precise_p1"], ost["impacted"]), (batch, kind, int(s))
