@@ -17,6 +17,10 @@
 
 #include "kernels.cuh"
 
+#ifndef CGB_PREREAD_CG
+#define CGB_PREREAD_CG 0
+#endif
+
 namespace cgb {
 
 namespace {
@@ -47,6 +51,9 @@ struct BParams {
     unsigned long long* stats;  // nullable: per query NSTAT counters
     uint32_t* err;
     uint32_t max_iters;
+    uint32_t bits_below;        // frontiers smaller than this keep a bitmap (else the masks M are scanned)
+    unsigned long long* trace;  // nullable: per iteration {t_start, t_s1, t_s2, phase<<62|q0<<32|listed, active<<32|edges}
+    uint32_t trace_cap;
 };
 
 // does row v hold a non-InitVal value for any query (and which)?
@@ -67,7 +74,7 @@ __device__ __forceinline__ uint32_t row_mask(const uint32_t* V, uint32_t v) {
 
 // ------------------------------------------------------------------ S1 (union frontier)
 template <int KIND, int B>
-__device__ void compact_b(const BParams& P, const GraphView& g, bool predicate, unsigned long long* cnt_slot,
+__device__ void compact_b(const BParams& P, const GraphView& g, bool predicate, bool from_m, unsigned long long* cnt_slot,
                           unsigned long long* act_slot, uint32_t* sm) {
     const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const uint64_t W = P.words;
@@ -86,6 +93,15 @@ __device__ void compact_b(const BParams& P, const GraphView& g, bool predicate, 
                 if (lane == j) word = bits;
             }
             if (wi < w1 && word) P.bitmap[wi] = word;
+        } else if (from_m) {  // union frontier = {v : M[v] != 0}: the last S2 set no bitmap bits
+#pragma unroll 8
+            for (uint32_t j = 0; j < 32; ++j) {
+                const uint32_t v = (g0 + j) * 32 + lane;
+                const bool act = g0 + j < w1 && v < P.n && ld_cg(P.M + v) != 0u;
+                const uint32_t bits = __ballot_sync(FULL, act);
+                if (lane == j) word = bits;
+            }
+            if (wi < w1) P.bitmap[wi] = word;
         } else if (wi < w1) {
             word = ld_cg(P.bitmap + wi);
         }
@@ -156,7 +172,7 @@ __device__ void compact_b(const BParams& P, const GraphView& g, bool predicate, 
                         mask = row_mask<KIND, B>(P.V, v);
                     } else {
                         mask = ld_cg(P.M + v);
-                        P.M[v] = 0u;  // consumed (deg-0 rows keep stale bits: they push nothing)
+                        P.M[v] = 0u;  // consumed
                     }
                 }
                 uint32_t incl = d;
@@ -189,9 +205,15 @@ struct Row {
 #pragma unroll
         for (int i = 0; i < B / 4; ++i) {
             uint4 t;
+#if CGB_PREREAD_CG
+            asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];"
+                         : "=r"(t.x), "=r"(t.y), "=r"(t.z), "=r"(t.w)
+                         : "l"(p + 4 * i));
+#else
             asm volatile("ld.global.ca.v4.u32 {%0,%1,%2,%3}, [%4];"
                          : "=r"(t.x), "=r"(t.y), "=r"(t.z), "=r"(t.w)
                          : "l"(p + 4 * i));
+#endif
             x[4 * i] = t.x;
             x[4 * i + 1] = t.y;
             x[4 * i + 2] = t.z;
@@ -212,7 +234,7 @@ struct Row {
 
 template <int KIND, bool PACKED, int B>
 __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, uint32_t E, uint32_t* xs /* 32*B */,
-                        uint32_t& n_edges, uint32_t& n_upd) {
+                        bool set_bits, uint32_t& n_edges, uint32_t& n_upd) {
     using O = Op<KIND>;
     constexpr int U = 2;  // edges per lane in flight
     const uint32_t lane = threadIdx.x & 31;
@@ -301,7 +323,7 @@ __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, ui
                 }
                 if (changed) {
                     red_or(P.M + d[u], changed);                              // v active for those queries
-                    red_or(P.bitmap + (d[u] >> 5), 1u << (d[u] & 31));        // v in the union frontier
+                    if (set_bits) red_or(P.bitmap + (d[u] >> 5), 1u << (d[u] & 31));  // union frontier bit
                 }
             }
         }
@@ -393,6 +415,7 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
 
         int phase = P.two_phase ? 1 : 2;
         bool predicate = false;
+        bool bits = true;  // the current frontier is in the bitmap (seeds set bits), else in M
         uint32_t iters = 0, n_edges = 0, n_upd = 0;  // (edge, query) pairs of the whole batch
         for (;;) {
             const GraphView& g = (phase == 1) ? P.C : P.G;
@@ -402,11 +425,21 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
                 unsigned long long* z = P.ctrl + CT0 + CTS * ((ring + 2) & 3);
                 z[0] = z[1] = 0ull;
             }
-            compact_b<KIND, B>(P, g, predicate, ctr + CT_LIST, ctr + CT_ACTIVE, sm_cnt);
+            const unsigned long long t_s0 = (P.trace && tid == 0) ? global_ns() : 0ull;
+            compact_b<KIND, B>(P, g, predicate, !bits, ctr + CT_LIST, ctr + CT_ACTIVE, sm_cnt);
             grid_sync(P.ctrl, epoch);
             ++ring;
             const unsigned long long ce = ld_cg64(ctr + CT_LIST);
             const uint32_t count = (uint32_t)(ce >> 32), E = (uint32_t)ce;
+            const uint32_t tr = ring - 1;
+            if (P.trace && tid == 0 && tr < P.trace_cap) {
+                unsigned long long* t = P.trace + 5ull * tr;
+                t[0] = t_s0;
+                t[1] = global_ns();
+                t[2] = 0;
+                t[3] = ((unsigned long long)phase << 62) | ((unsigned long long)q0 << 32) | count;
+                t[4] = (ld_cg64(ctr + CT_ACTIVE) << 32) | E;
+            }
             if (P.stats && tid == 0) {
                 const unsigned long long a = ld_cg64(ctr + CT_ACTIVE);
                 for (int b = 0; b < nq; ++b)  // union frontier, reported for every query of the batch
@@ -434,9 +467,13 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
                 }
                 break;
             }
-            relax_b<KIND, PACKED, B>(P, g, count, E, xs, n_edges, n_upd);
+            // small frontier: its S2 sets frontier bits (few reds) and the next S1 reads the bitmap;
+            // large frontier: no bitmap reds (they contend in L2), the next S1 scans M instead
+            bits = count < P.bits_below;
+            relax_b<KIND, PACKED, B>(P, g, count, E, xs, bits, n_edges, n_upd);
             predicate = false;
             grid_sync(P.ctrl, epoch);
+            if (P.trace && tid == 0 && tr < P.trace_cap) P.trace[5ull * tr + 2] = global_ns();
             if (++iters > P.max_iters) {
                 if (tid == 0) atomicOr(P.err, 1u);
                 return;
@@ -539,10 +576,22 @@ void run_queries_batched(Graph& G, const QueryCall& c, int B, cudaStream_t s, st
     P.stats = stats ? st.get() : nullptr;
     P.err = w.err.get();
     P.max_iters = G.n + 8;
+    {
+        const char* e = getenv("CG_BITS_BELOW");
+        P.bits_below = e ? (uint32_t)strtoul(e, nullptr, 10) : G.n / 256;
+    }
     CGB_CUDA(cudaMemsetAsync(w.bitmap.get(), 0, w.bitmap.bytes(), s));
     CGB_CUDA(cudaMemsetAsync(w.ctrl.get(), 0, w.ctrl.bytes(), s));
     CGB_CUDA(cudaMemsetAsync(w.err.get(), 0, 4, s));
     if (stats) CGB_CUDA(cudaMemsetAsync(st.get(), 0, st.bytes(), s));
+    static const bool tracing = getenv("CG_TRACE") != nullptr;
+    DevBuf<unsigned long long> trace;
+    if (tracing) {
+        P.trace_cap = 1u << 16;
+        trace.alloc(5ull * P.trace_cap, s);
+        CGB_CUDA(cudaMemsetAsync(trace.get(), 0, trace.bytes(), s));
+        P.trace = trace.get();
+    }
     if (G.packed) {
         if (B == 8) launch_kind_b<true, 8>(c.kind, P, G.num_sms, s);
         else if (B == 16) launch_kind_b<true, 16>(c.kind, P, G.num_sms, s);
@@ -551,6 +600,20 @@ void run_queries_batched(Graph& G, const QueryCall& c, int B, cudaStream_t s, st
         if (B == 8) launch_kind_b<false, 8>(c.kind, P, G.num_sms, s);
         else if (B == 16) launch_kind_b<false, 16>(c.kind, P, G.num_sms, s);
         else launch_kind_b<false, 32>(c.kind, P, G.num_sms, s);
+    }
+    if (tracing) {
+        std::vector<unsigned long long> h(5ull * P.trace_cap);
+        CGB_CUDA(cudaMemcpyAsync(h.data(), trace.get(), trace.bytes(), cudaMemcpyDeviceToHost, s));
+        CGB_CUDA(cudaStreamSynchronize(s));
+        unsigned long long t0 = 0;
+        for (uint32_t i = 0; i < P.trace_cap && h[5 * i]; ++i) {
+            const unsigned long long* t = h.data() + 5 * i;
+            if (!t0) t0 = t[0];
+            fprintf(stderr, "CG_TRACE kind=%d B=%d it=%u q0=%llu phase=%llu list=%llu active=%llu edges=%llu "
+                    "t=%.1f s1=%.1f s2=%.1f us\n", c.kind, B, i, (t[3] >> 32) & 0x3fffffffull, t[3] >> 62,
+                    t[3] & 0xffffffffull, t[4] >> 32, t[4] & 0xffffffffull, (t[0] - t0) / 1e3, (t[1] - t[0]) / 1e3,
+                    t[2] ? (t[2] - t[1]) / 1e3 : 0.0);
+        }
     }
     if (stats) {
         std::vector<unsigned long long> h((size_t)c.n_src * NSTAT);

@@ -265,3 +265,21 @@ def test_single_and_batched_engines(batch, monkeypatch):
             assert_values_equal(p1[i], op1, kind, f"B={batch} {kind} p1 s={s}")
             assert (st[i]["reached"], st[i]["precise_p1"], st[i]["impacted"]) == \
                 (ost["reached"], ost["precise_p1"], ost["impacted"]), (batch, kind, int(s))
+
+
+@pytest.mark.parametrize("bits_below", ["0", "4294967295"])
+def test_batched_frontier_modes(bits_below, monkeypatch):
+    """The batched engine keeps the union frontier either as bitmap bits set by S2 or as the
+    per-vertex query masks scanned by S1 (chosen per iteration); force each everywhere."""
+    monkeypatch.setenv("CG_BATCH", "16")
+    monkeypatch.setenv("CG_BITS_BELOW", bits_below)
+    n, m = 1 << 15, 16 << 15
+    src, dst, w = gen.rmat(n, m, w_max=15, seed=33)
+    g, og = both(n, src, dst, w)
+    sources = gen.sample_sources(n, src, dst, 20, seed=8)
+    for kind in ("sssp", "viterbi", "reach"):
+        g.build(kind, K=20)
+        for mode in ("2phase", "full"):
+            out = to_np(g.query(kind, to_dev(sources), mode=mode))
+            for i, s in enumerate(sources):
+                assert_values_equal(out[i], oracle.query(kind, og, int(s)), kind, f"bits<{bits_below} {kind} {mode}")

@@ -2,7 +2,7 @@
 # bench under several environment settings: tools/envbench.sh c2 "CG_BATCH=0" "CG_BATCH=8" ...
 cfg=$1; shift
 for envs in "$@"; do
-  tag=$(echo "$envs" | tr ' =' '__')
+  tag=$(echo "$envs" | sed "s|[^A-Za-z0-9_]|_|g" | tail -c 60)
   env $envs timeout 300 python bench.py --config $cfg --steps 5 --no-cpu-baseline --no-e2e > gpurun_out/eb_${cfg}_$tag.json 2> gpurun_out/eb_${cfg}_$tag.err
   python - "$cfg" "$tag" <<'PY'
 import json,sys
