@@ -17,9 +17,6 @@
 
 #include "kernels.cuh"
 
-#ifndef CGB_PREREAD_CG
-#define CGB_PREREAD_CG 0
-#endif
 
 namespace cgb {
 
@@ -52,6 +49,7 @@ struct BParams {
     uint32_t* err;
     uint32_t max_iters;
     uint32_t bits_below;        // frontiers smaller than this keep a bitmap (else the masks M are scanned)
+    uint32_t fresh;             // bit p-1: phase p pre-reads values from L2 instead of L1
     unsigned long long* trace;  // nullable: per iteration {t_start, t_s1, t_s2, phase<<62|q0<<32|listed, active<<32|edges}
     uint32_t trace_cap;
 };
@@ -201,19 +199,20 @@ __device__ void compact_b(const BParams& P, const GraphView& g, bool predicate, 
 template <int B>
 struct Row {
     uint32_t x[B];
-    __device__ void load_l1(const uint32_t* p) {  // Needed pre-read of all B values (may be stale)
+    // Needed pre-read of all B values: L1-allocating (may be stale, never better), or from L2
+    // (fresher: fewer redundant EdgeFunction atomics where values still change a lot)
+    __device__ void load(const uint32_t* p, bool fresh) {
 #pragma unroll
         for (int i = 0; i < B / 4; ++i) {
             uint4 t;
-#if CGB_PREREAD_CG
-            asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];"
-                         : "=r"(t.x), "=r"(t.y), "=r"(t.z), "=r"(t.w)
-                         : "l"(p + 4 * i));
-#else
-            asm volatile("ld.global.ca.v4.u32 {%0,%1,%2,%3}, [%4];"
-                         : "=r"(t.x), "=r"(t.y), "=r"(t.z), "=r"(t.w)
-                         : "l"(p + 4 * i));
-#endif
+            if (fresh)
+                asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];"
+                             : "=r"(t.x), "=r"(t.y), "=r"(t.z), "=r"(t.w)
+                             : "l"(p + 4 * i));
+            else
+                asm volatile("ld.global.ca.v4.u32 {%0,%1,%2,%3}, [%4];"
+                             : "=r"(t.x), "=r"(t.y), "=r"(t.z), "=r"(t.w)
+                             : "l"(p + 4 * i));
             x[4 * i] = t.x;
             x[4 * i + 1] = t.y;
             x[4 * i + 2] = t.z;
@@ -234,7 +233,7 @@ struct Row {
 
 template <int KIND, bool PACKED, int B>
 __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, uint32_t E, uint32_t* xs /* 32*B */,
-                        bool set_bits, uint32_t& n_edges, uint32_t& n_upd) {
+                        bool set_bits, bool fresh, uint32_t& n_edges, uint32_t& n_upd) {
     using O = Op<KIND>;
     constexpr int U = 2;  // edges per lane in flight
     const uint32_t lane = threadIdx.x & 31;
@@ -302,7 +301,7 @@ __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, ui
             for (int u = 0; u < U; ++u)
                 if (ok[u]) {
                     wd[u].decode(P.dbits, P.dmask, d[u], w[u]);
-                    cur[u].load_l1(P.V + (size_t)d[u] * B);
+                    cur[u].load(P.V + (size_t)d[u] * B, fresh);
                 }
 #pragma unroll
             for (int u = 0; u < U; ++u) {
@@ -470,7 +469,7 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
             // small frontier: its S2 sets frontier bits (few reds) and the next S1 reads the bitmap;
             // large frontier: no bitmap reds (they contend in L2), the next S1 scans M instead
             bits = count < P.bits_below;
-            relax_b<KIND, PACKED, B>(P, g, count, E, xs, bits, n_edges, n_upd);
+            relax_b<KIND, PACKED, B>(P, g, count, E, xs, bits, (P.fresh >> (phase - 1)) & 1u, n_edges, n_upd);
             predicate = false;
             grid_sync(P.ctrl, epoch);
             if (P.trace && tid == 0 && tr < P.trace_cap) P.trace[5ull * tr + 2] = global_ns();
@@ -579,6 +578,8 @@ void run_queries_batched(Graph& G, const QueryCall& c, int B, cudaStream_t s, st
     {
         const char* e = getenv("CG_BITS_BELOW");
         P.bits_below = e ? (uint32_t)strtoul(e, nullptr, 10) : G.n / 256;
+        const char* f = getenv("CG_FRESH");
+        P.fresh = f ? (uint32_t)strtoul(f, nullptr, 10) : 0u;
     }
     CGB_CUDA(cudaMemsetAsync(w.bitmap.get(), 0, w.bitmap.bytes(), s));
     CGB_CUDA(cudaMemsetAsync(w.ctrl.get(), 0, w.ctrl.bytes(), s));
