@@ -137,28 +137,39 @@ def host_edges(cfg):
     return gen.rmat(cfg.n, cfg.m, cfg.abcd, cfg.w_max, cfg.seed)
 
 
-def sources_for(cfg, src_h, dst_h, kind_idx, count, rank, world=1):
+def sources_for(cand, kind_idx, count, rank, world=1):
     """Rank's contiguous shard of the kind's global seeded source list (count per rank: weak
-    scaling over independent vertex queries)."""
+    scaling over independent vertex queries).  cand = gen.source_candidates(...)."""
     import gen
     from paper_conf_eurosys_0002a0a024_b200 import multi
-    allsrc = gen.sample_sources(cfg.n, src_h, dst_h, count * world, seed=1000 + 17 * kind_idx)
+    allsrc = gen.sample_from(cand, count * world, seed=1000 + 17 * kind_idx)
     a, b = multi.shard(len(allsrc), rank, world)
     return allsrc[a:b]
+
+
+def device_candidates(n, src_d, dst_d):
+    """gen.source_candidates computed on the device twin's (bit-identical) raw edge list."""
+    import torch
+    has = torch.zeros(n, dtype=torch.bool, device=src_d.device)
+    keep = src_d.view(torch.int32) != dst_d.view(torch.int32)
+    has[src_d.view(torch.int32)[keep].to(torch.int64)] = True
+    return torch.nonzero(has).flatten().to(torch.int64).cpu().numpy().astype(np.uint32)
 
 
 # ---------------------------------------------------------------------------- CPU oracle arm
 def cpu_oracle_run(cfg, src_h, dst_h, w_h, kinds, per_kind, rank=0):
     """Time the oracle (as it stands: label-setting Dijkstra per kind, one source per OpenMP
     thread) on a bounded sample of the same workload.  Returns (queries/s, cores, sample, og)."""
+    import gen
     import oracle
     t0 = time.time()
     og = oracle.canonical_csr(cfg.n, src_h, dst_h, w_h)
+    cand = gen.source_candidates(cfg.n, src_h, dst_h)
     build_s = time.time() - t0
     cores = os.cpu_count() or 1
     total_q, total_t = 0, 0.0
     for ki, kind in enumerate(kinds):
-        srcs = sources_for(cfg, src_h, dst_h, KINDS.index(kind), per_kind, rank)
+        srcs = sources_for(cand, KINDS.index(kind), per_kind, rank)
         t0 = time.perf_counter()
         oracle.query_batch(kind, og, srcs, nthreads=cores)
         total_t += time.perf_counter() - t0
@@ -217,10 +228,15 @@ def main():
     if args.warmup < 3:
         args.warmup = 3  # timing rule: >= 3 warm-up steps
 
-    # ---- inputs (untimed): host edges for sources / oracle, device twin for the graph
+    # ---- inputs (untimed): the device twin of the generator for the graph and the source
+    # candidates; host edges only for the oracle's cpu_baseline (rank 0, N = 1)
     t0 = time.time()
-    src_h, dst_h, w_h = host_edges(cfg)
+    need_host = rank == 0 and ws == 1 and not args.no_cpu_baseline
+    src_h = dst_h = w_h = None
+    if need_host:
+        src_h, dst_h, w_h = host_edges(cfg)
     src_d, dst_d, w_d = rmat_device(cfg.n, cfg.m, cfg.abcd, cfg.w_max, cfg.seed, True, dev)
+    cand = device_candidates(cfg.n, src_d, dst_d)
     g = Graph(cfg.n, src_d, dst_d, w_d, device=dev)
     del src_d, dst_d, w_d
     torch.cuda.synchronize()
@@ -231,10 +247,10 @@ def main():
             build["bfs"] = dict(build["reach"])
             continue
         build[kind] = g.build(kind, K=args.K)
-    ptr, _, _ = g.export()
+    ptr = g.export(ptr_only=True)[0]
     outdeg = (ptr[1:] - ptr[:-1]).to(torch.int64)
     del ptr
-    srcs = {k: torch.from_numpy(sources_for(cfg, src_h, dst_h, KINDS.index(k), B, rank, ws).astype(np.int64))
+    srcs = {k: torch.from_numpy(sources_for(cand, KINDS.index(k), B, rank, ws).astype(np.int64))
             .to(torch.uint32).to(dev) for k in kinds}
     nbuf = 2 if gather else 1
     outs = [{k: torch.empty((B, cfg.n), dtype=torch.uint32, device=dev) for k in kinds} for _ in range(nbuf)]

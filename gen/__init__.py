@@ -125,19 +125,24 @@ CONFIGS = {
 }
 
 
-def sample_sources(n: int, src: np.ndarray, dst: np.ndarray, count: int, seed: int) -> np.ndarray:
-    """Uniform sources over vertices with outdeg > 0, seeded, distinct when possible.
-
-    Computed from the RAW edge list: a vertex has a non-self-loop out-edge in
-    the raw list iff it has outdeg > 0 after canonicalization, so neither
-    side's CSR is needed to draw the sources.
-    """
+def source_candidates(n: int, src: np.ndarray, dst: np.ndarray) -> np.ndarray:
+    """Sorted ids of the vertices with a non-self-loop out-edge in the RAW edge list: exactly the
+    vertices with outdeg > 0 after canonicalization, so neither side's CSR is needed."""
     has_out = np.zeros(n, dtype=bool)
     keep = src != dst
     has_out[src[keep]] = True
-    cand = np.nonzero(has_out)[0].astype(np.uint32)
+    return np.nonzero(has_out)[0].astype(np.uint32)
+
+
+def sample_from(cand: np.ndarray, count: int, seed: int) -> np.ndarray:
+    """`count` sources drawn uniformly from `cand`, seeded, distinct when possible."""
     if cand.size == 0:
         return np.zeros(0, dtype=np.uint32)
     rng = np.random.default_rng(seed)
     replace = count > cand.size
     return np.sort(rng.choice(cand, size=count, replace=replace)).astype(np.uint32)
+
+
+def sample_sources(n: int, src: np.ndarray, dst: np.ndarray, count: int, seed: int) -> np.ndarray:
+    """Uniform sources over vertices with outdeg > 0, seeded, distinct when possible."""
+    return sample_from(source_candidates(n, src, dst), count, seed)

@@ -108,8 +108,8 @@ cg_status cg_graph_destroy(cg_graph g);
 cg_status cg_graph_info(cg_graph g, int64_t* n, int64_t* m, uint32_t* w_max);
 
 /* Copy the canonical CSR (transpose = 0) or CSC (transpose = 1) into caller device buffers:
- * ptr int64[n+1], idx uint32[m] (destinations for CSR, sources for CSC), w uint32[m].
- * Stream-ordered. */
+ * ptr int64[n+1], idx uint32[m] (destinations for CSR, sources for CSC), w uint32[m]; idx and
+ * w may both be NULL to copy the row offsets only.  Stream-ordered. */
 cg_status cg_graph_export(cg_graph g, int transpose, int64_t* ptr, uint32_t* idx, uint32_t* w, void* stream);
 
 /*

@@ -163,7 +163,7 @@ cg_status cg_graph_info(cg_graph g, int64_t* n, int64_t* m, uint32_t* w_max) {
 cg_status cg_graph_export(cg_graph g, int transpose, int64_t* ptr, uint32_t* idx, uint32_t* w, void* stream) {
     return guard([&] {
         CGB_CHECK(g != nullptr, CG_EINVAL, "null graph");
-        CGB_CHECK(ptr && (g->G.m == 0 || (idx && w)), CG_EINVAL, "null output");
+        CGB_CHECK(ptr && (idx != nullptr) == (w != nullptr), CG_EINVAL, "null output");
         CGB_CUDA(cudaSetDevice(g->G.device));
         export_adj(g->G, transpose ? g->G.gr : g->G.g, ptr, idx, w, S(stream));
     });

@@ -123,7 +123,7 @@ __global__ void k_export(uint32_t n, uint32_t m, uint32_t dbits, const uint32_t*
     uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
     for (uint64_t i = t; i <= n; i += stride) ptr[i] = ptr32[i];
     uint32_t mask = dbits >= 32 ? 0xffffffffu : ((1u << dbits) - 1u);
-    for (uint64_t i = t; i < m; i += stride) {
+    for (uint64_t i = t; idx && i < m; i += stride) {
         uint32_t d, ww;
         if (adj) { uint32_t x = adj[i]; d = x & mask; ww = (x >> dbits) + 1u; }
         else { uint2 x = adjw[i]; d = x.x; ww = x.y; }

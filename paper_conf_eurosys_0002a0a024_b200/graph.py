@@ -111,11 +111,12 @@ class Graph:
         self.close()
 
     # -------------------------------------------------------------- graph
-    def export(self, transpose: bool = False):
-        """(ptr int64[n+1], idx uint32[m], w uint32[m]) of the canonical CSR (or CSC)."""
+    def export(self, transpose: bool = False, ptr_only: bool = False):
+        """(ptr int64[n+1], idx uint32[m], w uint32[m]) of the canonical CSR (or CSC); with
+        ptr_only the edge arrays are not copied (returned as None)."""
         ptr = torch.empty(self.n + 1, dtype=torch.int64, device=self.device)
-        idx = torch.empty(self.m, dtype=torch.uint32, device=self.device)
-        w = torch.empty(self.m, dtype=torch.uint32, device=self.device)
+        idx = None if ptr_only else torch.empty(self.m, dtype=torch.uint32, device=self.device)
+        w = None if ptr_only else torch.empty(self.m, dtype=torch.uint32, device=self.device)
         with torch.cuda.device(self.device):
             _lib.call("cg_graph_export", self._h, 1 if transpose else 0, _ptr(ptr), _ptr(idx), _ptr(w),
                       _stream(self.device))
