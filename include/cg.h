@@ -61,8 +61,9 @@ typedef enum { CG_HUBS_TOPDEG = 0, CG_HUBS_SAMPLED = 1, CG_HUBS_GIVEN = 2 } cg_h
 
 /* Which Core Graph construction: AUTO = Algorithm 1 (specialized) for
  * SSSP/SSWP/SSNP/VITERBI and Algorithm 2 (general) for BFS/REACH
- * (reading Q12). */
-typedef enum { CG_ALG_AUTO = 0, CG_ALG_SPECIALIZED = 1, CG_ALG_GENERAL = 2 } cg_cg_alg;
+ * (reading Q12).  GENERAL uses one Qid[] for both traversal directions (the
+ * literal Alg 2, reading Q9); GENERAL_PERDIR keeps one Qid[] per direction. */
+typedef enum { CG_ALG_AUTO = 0, CG_ALG_SPECIALIZED = 1, CG_ALG_GENERAL = 2, CG_ALG_GENERAL_PERDIR = 3 } cg_cg_alg;
 
 typedef struct cg_graph_s* cg_graph; /* opaque: owns G (CSR), G^R (CSC) and the CGs on one device */
 

@@ -224,10 +224,11 @@ def full_bsp(kind, g: CSR, s: int):
 
 
 def cg_for_kind(kind, g: CSR, gr: CSR, hubs) -> np.ndarray:
-    """The CG each kind uses (reading A12/Q12): Alg 1 for SSSP/SSWP/SSNP/Viterbi, Alg 2 for BFS/REACH."""
+    """The CG each kind uses by default (readings Q12, Q9'): Alg 1 for SSSP/SSWP/SSNP/Viterbi,
+    Alg 2 with one Qid[] per traversal direction for BFS/REACH (reading Q9')."""
     k = _kind(kind)
     if k in (KINDS["bfs"], KINDS["reach"]):
-        return cg_alg2(g, gr, hubs)
+        return cg_alg2(g, gr, hubs, per_direction=True)
     return cg_alg1(k, g, gr, hubs)
 
 

@@ -304,8 +304,29 @@ void mark_group(Graph& G, int nh, const uint32_t* vf, const uint32_t* vb, uint8_
     CGB_LAUNCH(k_mark_tight<KIND>, grid_rows(G.n), TB, 0, s, G.n, view(G.g), G.dbits, nh, vf, vb, flags);
 }
 
-void alg1(Graph& G, int kind, const std::vector<uint32_t>& hubs, uint8_t* flags, cudaStream_t s) {
+// hub rows for the NEXT-1 certificates (row stride 2*KP, KP = K rounded up to 4 so that the
+// engine reads 16 B chunks): HB[v][k0+j] = vf[j][v], HB[v][KP+k0+j] = vb[j][v]
+__global__ void k_hub_rows(uint32_t n, int nh, int k0, int KP, const uint32_t* __restrict__ vf,
+                           const uint32_t* __restrict__ vb, uint32_t* __restrict__ hb) {
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < (uint64_t)n * nh;
+         i += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t j = (uint32_t)(i / n), v = (uint32_t)(i % n);
+        hb[(size_t)v * 2 * KP + k0 + j] = vf[(size_t)j * n + v];
+        hb[(size_t)v * 2 * KP + KP + k0 + j] = vb[(size_t)j * n + v];
+    }
+}
+
+void alg1(Graph& G, int kind, const std::vector<uint32_t>& hubs, uint8_t* flags, Core& C, cudaStream_t s) {
     const int K = (int)hubs.size();
+    // certificates are kept for the kinds that have one (SSSP, SSWP, SSNP) and K <= 64
+    const bool keep = (kind == CG_SSSP || kind == CG_SSWP || kind == CG_SSNP) && K <= 64;
+    C.hub_vals.reset();
+    C.hub_k = 0;
+    const int KP = (K + 3) & ~3;
+    if (keep) {
+        C.hub_vals.alloc((size_t)G.n * 2 * KP, s);
+        C.hub_k = (uint32_t)K;
+    }
     const int group = K < 16 ? K : 16;
     DevBuf<uint32_t> hsrc(K, s);
     CGB_CUDA(cudaMemcpyAsync(hsrc.get(), hubs.data(), 4ull * K, cudaMemcpyHostToDevice, s));
@@ -324,19 +345,24 @@ void alg1(Graph& G, int kind, const std::vector<uint32_t>& hubs, uint8_t* flags,
         case CG_BFS: mark_group<CG_BFS>(G, nh, vf.get(), vb.get(), flags, s); break;
         case CG_REACH: mark_group<CG_REACH>(G, nh, vf.get(), vb.get(), flags, s); break;
         }
+        if (keep)
+            CGB_LAUNCH(k_hub_rows, 4096, TB, 0, s, G.n, nh, k0, KP, vf.get(), vb.get(), C.hub_vals.get());
     }
 }
 
-void alg2(Graph& G, const std::vector<uint32_t>& hubs, uint8_t* flags, cudaStream_t s) {
+void alg2(Graph& G, const std::vector<uint32_t>& hubs, uint8_t* flags, bool per_direction, cudaStream_t s) {
     const uint32_t n = G.n;
-    DevBuf<uint32_t> qid(n, s), la(n + 1, s), lb(n + 1, s), cnt(n + 1, s), base(n + 1, s);
+    // reading Q9: one Qid[] shared by the forward and backward traversals (literal Alg 2), or
+    // one per direction (CG_ALG_GENERAL_PERDIR)
+    DevBuf<uint32_t> qid(per_direction ? 2ull * n : n, s), la(n + 1, s), lb(n + 1, s), cnt(n + 1, s), base(n + 1, s);
     DevBuf<unsigned long long> key(n, s);
-    CGB_CUDA(cudaMemsetAsync(qid.get(), 0, 4ull * n, s));
+    CGB_CUDA(cudaMemsetAsync(qid.get(), 0, qid.bytes(), s));
     CGB_CUDA(cudaMemsetAsync(key.get(), 0xff, 8ull * n, s));
     for (size_t k = 0; k < hubs.size(); ++k) {               // Alg 2 l.5
         const uint32_t lab = (uint32_t)k + 1;                 // reading Q10
         for (int dir = 0; dir < 2; ++dir) {                   // l.6 on G, l.7 on G^R
             const GraphView g = dir == 0 ? view(G.g) : view(G.gr);
+            uint32_t* Q = qid.get() + (per_direction && dir == 1 ? n : 0);
             uint32_t* L = la.get();
             uint32_t* N = lb.get();
             uint32_t nl = 1;
@@ -344,15 +370,15 @@ void alg2(Graph& G, const std::vector<uint32_t>& hubs, uint8_t* flags, cudaStrea
             while (nl) {                                                          // l.13
                 const int grid = grid_rows(nl);
                 if (dir == 0) {
-                    CGB_LAUNCH(k_alg2_expand<false>, grid, TB, 0, s, g, G.dbits, L, nl, qid.get(), lab, key.get(),
+                    CGB_LAUNCH(k_alg2_expand<false>, grid, TB, 0, s, g, G.dbits, L, nl, Q, lab, key.get(),
                                flags, (const uint32_t*)nullptr);
-                    CGB_LAUNCH((k_alg2_winners<false, false>), grid, TB, 0, s, g, G.dbits, L, nl, qid.get(), lab,
+                    CGB_LAUNCH((k_alg2_winners<false, false>), grid, TB, 0, s, g, G.dbits, L, nl, Q, lab,
                                key.get(), cnt.get(), (const uint32_t*)nullptr, (uint32_t*)nullptr, flags,
                                (const uint32_t*)nullptr);
                 } else {
-                    CGB_LAUNCH(k_alg2_expand<true>, grid, TB, 0, s, g, G.dbits, L, nl, qid.get(), lab, key.get(),
+                    CGB_LAUNCH(k_alg2_expand<true>, grid, TB, 0, s, g, G.dbits, L, nl, Q, lab, key.get(),
                                flags, G.reid.get());
-                    CGB_LAUNCH((k_alg2_winners<false, true>), grid, TB, 0, s, g, G.dbits, L, nl, qid.get(), lab,
+                    CGB_LAUNCH((k_alg2_winners<false, true>), grid, TB, 0, s, g, G.dbits, L, nl, Q, lab,
                                key.get(), cnt.get(), (const uint32_t*)nullptr, (uint32_t*)nullptr, flags,
                                G.reid.get());
                 }
@@ -363,10 +389,10 @@ void alg2(Graph& G, const std::vector<uint32_t>& hubs, uint8_t* flags, cudaStrea
                 CGB_CUDA(cudaStreamSynchronize(s));
                 if (total) {
                     if (dir == 0)
-                        CGB_LAUNCH((k_alg2_winners<true, false>), grid, TB, 0, s, g, G.dbits, L, nl, qid.get(), lab,
+                        CGB_LAUNCH((k_alg2_winners<true, false>), grid, TB, 0, s, g, G.dbits, L, nl, Q, lab,
                                    key.get(), cnt.get(), base.get(), N, flags, (const uint32_t*)nullptr);
                     else
-                        CGB_LAUNCH((k_alg2_winners<true, true>), grid, TB, 0, s, g, G.dbits, L, nl, qid.get(), lab,
+                        CGB_LAUNCH((k_alg2_winners<true, true>), grid, TB, 0, s, g, G.dbits, L, nl, Q, lab,
                                    key.get(), cnt.get(), base.get(), N, flags, G.reid.get());
                 }
                 uint32_t* t = L; L = N; N = t;
@@ -382,9 +408,11 @@ void build_core(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs_
                 int connectivity, cudaStream_t s) {
     CGB_CHECK(kind >= 0 && kind <= CG_REACH, CG_EINVAL, "bad kind");
     CGB_CHECK(K > 0 && (uint32_t)K <= G.n, CG_EINVAL, "K must be in [1, n]");
-    if (alg == CG_ALG_AUTO) alg = (kind == CG_BFS || kind == CG_REACH) ? CG_ALG_GENERAL : CG_ALG_SPECIALIZED;
-    CGB_CHECK(alg == CG_ALG_SPECIALIZED || alg == CG_ALG_GENERAL, CG_EINVAL, "bad CG algorithm");
-    if (connectivity < 0) connectivity = (alg == CG_ALG_SPECIALIZED) ? 1 : 0;
+    // reading Q9': the general CG keeps one Qid[] per traversal direction by default
+    if (alg == CG_ALG_AUTO) alg = (kind == CG_BFS || kind == CG_REACH) ? CG_ALG_GENERAL_PERDIR : CG_ALG_SPECIALIZED;
+    CGB_CHECK(alg == CG_ALG_SPECIALIZED || alg == CG_ALG_GENERAL || alg == CG_ALG_GENERAL_PERDIR, CG_EINVAL,
+              "bad CG algorithm");
+    if (connectivity < 0) connectivity = (alg == CG_ALG_SPECIALIZED) ? 1 : 0;  // reading Q11
 
     cudaEvent_t e0, e1;
     CGB_CUDA(cudaEventCreate(&e0));
@@ -394,11 +422,13 @@ void build_core(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs_
     std::vector<uint32_t> hubs = select_hubs(G, K, policy, hubs_in, seed, s);
     Core& C = G.core[core_slot(kind)];
     C.built = false;
+    C.hub_vals.reset();
+    C.hub_k = 0;
     C.flags.alloc(G.m ? G.m : 1, s);
     CGB_CUDA(cudaMemsetAsync(C.flags.get(), 0, C.flags.bytes(), s));
     if (G.m) {
-        if (alg == CG_ALG_SPECIALIZED) alg1(G, kind, hubs, C.flags.get(), s);
-        else alg2(G, hubs, C.flags.get(), s);
+        if (alg == CG_ALG_SPECIALIZED) alg1(G, kind, hubs, C.flags.get(), C, s);
+        else alg2(G, hubs, C.flags.get(), alg == CG_ALG_GENERAL_PERDIR, s);
         if (connectivity) {
             const int sel = (kind == CG_SSWP) ? 1 : ((kind == CG_BFS || kind == CG_REACH) ? 2 : 0);
             CGB_LAUNCH(k_connectivity, grid_rows(G.n), TB, 0, s, G.n, view(G.g), G.dbits, sel, C.flags.get());

@@ -49,6 +49,10 @@ struct BParams {
     uint32_t* err;
     uint32_t max_iters;
     uint32_t bits_below;        // frontiers smaller than this keep a bitmap (else the masks M are scanned)
+    GraphView R;                // G^R: in-edges for the NEXT-1 pull
+    const uint32_t* HB;         // CG hub rows [n][2K] for the certificates (nullable)
+    uint32_t K, KP;             // hubs in HB; row stride 2*KP (KP = K rounded up to a multiple of 4)
+    int reduced;                // phase 2 starts with the certificate-driven pull (NEXT-1)
     uint32_t fresh;             // bit p-1: phase p pre-reads values from L2 instead of L1
     unsigned long long* trace;  // nullable: per iteration {t_start, t_s1, t_s2, phase<<62|q0<<32|listed, active<<32|edges}
     uint32_t trace_cap;
@@ -70,10 +74,83 @@ __device__ __forceinline__ uint32_t row_mask(const uint32_t* V, uint32_t v) {
     return m;
 }
 
-// ------------------------------------------------------------------ S1 (union frontier)
+// ------------------------------------------------------------------ NEXT-1 certificates
+// p = Val(s,v) after phase 1 on the CG, a bound on the true value from the "worse" side.
+// Fv/Rv = Q(h) on G / on G^R at v, Fs/Rs the same at the source.  A certificate is a bound
+// from the other side, met with equality (Theorem 1; bottleneck analogs):
+//   SSWP (p <= W(s,v)): W(v,h) > W(s,h) => W(s,v) <= W(s,h);  W(h,s) > W(h,v) => W(s,v) <= W(h,v)
+//   SSNP (p >= N(s,v)): N(v,h) < N(s,h) => N(s,v) >= N(s,h);  N(h,s) < N(h,v) => N(s,v) >= N(h,v)
+//   SSSP (p >= d(s,v)): d(s,v) >= d(s,h) - d(v,h);  d(s,v) >= d(h,v) - d(h,s)  (Theorem 1), with
+//        "infinite minus finite" = infinite (s cannot reach v when v reaches h but s does not, ...)
+template <int KIND>
+__device__ __forceinline__ bool certified(uint32_t p, uint32_t Fv, uint32_t Rv, uint32_t Fs, uint32_t Rs) {
+    if (KIND == CG_SSWP) return (Rv > Rs && p == Rs) || (Fs > Fv && p == Fv);
+    if (KIND == CG_SSNP) return (Rv < Rs && p == Rs) || (Fs < Fv && p == Fv);
+    if (KIND == CG_SSSP) {
+        constexpr uint32_t INF = 0xffffffffu;
+        if (Rv != INF && p == (Rs == INF ? INF : (Rs > Rv ? Rs - Rv : 0u))) return true;
+        if (Fs != INF && p == (Fv == INF ? INF : (Fv > Fs ? Fv - Fs : 0u))) return true;
+    }
+    return false;
+}
+
+// queries q < nq whose phase-1 value at v is not proven final (Reduced(E) keeps v's in-edges).
+// Kept register-light (it runs inside the persistent kernel): the value row is only compared,
+// then each open query re-reads its value and scans the hub row 4 hubs per 16 B load.
 template <int KIND, int B>
-__device__ void compact_b(const BParams& P, const GraphView& g, bool predicate, bool from_m, unsigned long long* cnt_slot,
-                          unsigned long long* act_slot, uint32_t* sm) {
+__device__ uint32_t uncertified(const BParams& P, const uint32_t* sh, int nq, uint32_t v) {
+    using O = Op<KIND>;
+    const uint32_t* row = P.V + (size_t)v * B;
+    uint32_t unc = 0;
+#pragma unroll
+    for (int i = 0; i < B / 4; ++i) {
+        uint4 x;
+        asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];"
+                     : "=r"(x.x), "=r"(x.y), "=r"(x.z), "=r"(x.w)
+                     : "l"(reinterpret_cast<const uint4*>(row) + i));
+        unc |= (uint32_t)(x.x != O::SRC) << (4 * i) | (uint32_t)(x.y != O::SRC) << (4 * i + 1) |
+               (uint32_t)(x.z != O::SRC) << (4 * i + 2) | (uint32_t)(x.w != O::SRC) << (4 * i + 3);
+    }
+    unc &= nq >= 32 ? 0xffffffffu : ((1u << nq) - 1u);  // the lattice top (REACH: reached) is final
+    if (KIND == CG_REACH || P.HB == nullptr || !unc) return unc;
+    // hub row of v: F at [0, KP), R at [KP, 2 KP) (KP = K rounded up to 4: 16 B aligned chunks)
+    const uint32_t K = P.K, KP = P.KP;
+    const uint4* hb = reinterpret_cast<const uint4*>(P.HB + (size_t)v * 2 * KP);
+    uint32_t todo = unc;
+    while (todo) {
+        const int q = __ffs(todo) - 1;
+        todo &= todo - 1;
+        const uint32_t p = ld_cg(row + q);
+        const uint32_t* sq = sh + q * 2 * K;
+        for (uint32_t h0 = 0; h0 < K; h0 += 4) {
+            const uint4 f = __ldg(hb + h0 / 4), r = __ldg(hb + (KP + h0) / 4);
+            bool c = false;
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                const uint32_t h = h0 + j;
+                const uint32_t Fv = j == 0 ? f.x : j == 1 ? f.y : j == 2 ? f.z : f.w;
+                const uint32_t Rv = j == 0 ? r.x : j == 1 ? r.y : j == 2 ? r.z : r.w;
+                c |= h < K && certified<KIND>(p, Fv, Rv, sq[h], sq[K + h]);
+            }
+            if (c) {
+                unc &= ~(1u << q);
+                break;
+            }
+        }
+    }
+    return unc;
+}
+
+// ------------------------------------------------------------------ S1 (union frontier)
+// mode: F_BITS (frontier bits set by S2), F_MASKS (frontier = {v : M[v] != 0}), F_IMPACTED
+// (Alg 3 l.15: v active for q iff Val(v) != InitVal), F_UNCERT (NEXT-1: v active for its
+// uncertified queries; degrees are then in-degrees, g = G^R).
+enum { F_BITS = 0, F_MASKS = 1, F_IMPACTED = 2, F_UNCERT = 3 };
+
+template <int KIND, int B>
+__device__ void compact_b(const BParams& P, const GraphView& g, int mode, const uint32_t* sh, int nq,
+                          unsigned long long* cnt_slot, unsigned long long* act_slot, uint32_t* sm) {
+    const bool predicate = mode == F_IMPACTED;
     const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const uint64_t W = P.words;
     const uint32_t w0 = (uint32_t)(W * blockIdx.x / gridDim.x), w1 = (uint32_t)(W * (blockIdx.x + 1) / gridDim.x);
@@ -91,7 +168,16 @@ __device__ void compact_b(const BParams& P, const GraphView& g, bool predicate, 
                 if (lane == j) word = bits;
             }
             if (wi < w1 && word) P.bitmap[wi] = word;
-        } else if (from_m) {  // union frontier = {v : M[v] != 0}: the last S2 set no bitmap bits
+        } else if (mode == F_UNCERT) {  // certificates: the uncertified queries' mask parks in M
+            for (uint32_t j = 0; j < 32; ++j) {
+                const uint32_t v = (g0 + j) * 32 + lane;
+                const uint32_t unc = (g0 + j < w1 && v < P.n) ? uncertified<KIND, B>(P, sh, nq, v) : 0u;
+                if (unc) P.M[v] = unc;
+                const uint32_t bits = __ballot_sync(FULL, unc != 0);
+                if (lane == j) word = bits;
+            }
+            if (wi < w1) P.bitmap[wi] = word;
+        } else if (mode == F_MASKS) {  // union frontier = {v : M[v] != 0}: the last S2 set no bitmap bits
 #pragma unroll 8
             for (uint32_t j = 0; j < 32; ++j) {
                 const uint32_t v = (g0 + j) * 32 + lane;
@@ -332,6 +418,108 @@ __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, ui
     }
 }
 
+// ------------------------------------------------------------------ NEXT-1 pull (Reduced(E))
+// The list holds vertices v with uncertified queries (mask) and their IN-edge offsets; a lane
+// takes an in-edge (u -> v, w) of the edge-balanced split and, for each uncertified query q
+// with Val(u) reached, applies the Table 6 Needed / EdgeFunction to Val(v): all pushes INTO
+// uncertified vertices in one sweep, none into certified ones (their in-edges are removed).
+template <int KIND, bool PACKED, int B>
+__device__ void relax_pull(const BParams& P, uint32_t count, uint32_t E, uint32_t* xs, uint32_t& n_edges,
+                           uint32_t& n_upd) {
+    using O = Op<KIND>;
+    constexpr int U = 2;
+    const GraphView& g = P.R;
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t gw = blockIdx.x * BW + (threadIdx.x >> 5);
+    const uint64_t NW = (uint64_t)gridDim.x * BW;
+    const uint32_t e0 = (uint32_t)((uint64_t)E * gw / NW), e1 = (uint32_t)((uint64_t)E * (gw + 1) / NW);
+    if (e0 >= e1) return;
+    uint32_t lo = 0, hi = count;
+    while (hi - lo > 32) {
+        const uint32_t step = (hi - lo + 31) / 32;
+        const uint32_t p = lo + lane * step;
+        const bool le = p < hi && ld_cg(P.lo + p) <= e0;
+        const uint32_t k = 31 - __clz(__ballot_sync(FULL, le));
+        const uint32_t nlo = lo + k * step;
+        hi = min(hi, nlo + step);
+        lo = nlo;
+    }
+    {
+        const uint32_t p = lo + lane;
+        const bool le = p < hi && ld_cg(P.lo + p) <= e0;
+        lo += 31 - __clz(__ballot_sync(FULL, le));
+    }
+    uint32_t i = lo, e = e0;
+    for (;;) {
+        const uint32_t idx = i + lane;
+        uint32_t off = E, base = 0, v = 0, mask = 0;
+        if (idx < count) {
+            v = ld_cg(P.lv + idx);
+            off = ld_cg(P.lo + idx);
+            mask = ld_cg(P.lm + idx);
+            base = __ldg(g.ptr + v) - off;
+        }
+        __syncwarp();
+#pragma unroll
+        for (int r = 0; r < B; ++r) {  // current rows of the pulling vertices (for the Needed test)
+            const uint32_t f = r * 32 + lane;
+            const uint32_t vr = __shfl_sync(FULL, v, f / B);
+            xs[f] = (i + f / B < count) ? ld_cg(P.V + (size_t)vr * B + f % B) : 0u;
+        }
+        __syncwarp();
+        const uint32_t wend = (i + 32 < count) ? ld_cg(P.lo + i + 32) : E;
+        const uint32_t ehi = min(e1, wend);
+        for (; e < ehi; e += 32 * U) {
+            uint32_t k[U], mk[U], vk[U];
+            bool ok[U];
+            EdgeWord<PACKED> wd[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                const uint32_t t = e + u * 32 + lane;
+                uint32_t kk = 0;
+#pragma unroll
+                for (uint32_t st = 16; st > 0; st >>= 1)
+                    if (__shfl_sync(FULL, off, kk + st) <= t) kk += st;
+                k[u] = kk;
+                mk[u] = __shfl_sync(FULL, mask, kk);
+                vk[u] = __shfl_sync(FULL, v, kk);
+                const uint32_t a = __shfl_sync(FULL, base, kk) + t;
+                ok[u] = t < ehi;
+                if (ok[u]) wd[u].load(g, a);
+            }
+            uint32_t src[U], w[U];
+            Row<B> xu[U];
+#pragma unroll
+            for (int u = 0; u < U; ++u)
+                if (ok[u]) {
+                    wd[u].decode(P.dbits, P.dmask, src[u], w[u]);
+                    xu[u].load(P.V + (size_t)src[u] * B, false);
+                }
+#pragma unroll
+            for (int u = 0; u < U; ++u) {
+                if (!ok[u]) continue;
+                uint32_t changed = 0;
+#pragma unroll
+                for (int q = 0; q < B; ++q) {
+                    if (!((mk[u] >> q) & 1u)) continue;
+                    ++n_edges;
+                    if (xu[u].x[q] == O::INIT) continue;  // u unreached for q: nothing to pull
+                    const uint32_t cand = O::ext(xu[u].x[q], w[u]);
+                    if (O::better(cand, xs[k[u] * B + q])) {              // Needed(e(u,v)), query q
+                        O::edge_fn(P.V + (size_t)vk[u] * B + q, cand);    // EdgeFunction
+                        changed |= 1u << q;
+                        ++n_upd;
+                    }
+                }
+                if (changed) red_or(P.M + vk[u], changed);  // v pushes onward for those queries
+            }
+        }
+        if (ehi >= e1) break;
+        e = ehi;
+        i += 32;
+    }
+}
+
 // Batch-total count c (per thread) split evenly over the nq queries' counter k: block sum,
 // then thread 0 adds total/nq to each (the remainder to the first).
 __device__ __forceinline__ void block_add_split(unsigned long long* stats, int q0, int nq, int k, unsigned long long c,
@@ -378,8 +566,9 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
     using O = Op<KIND>;
     __shared__ uint32_t sm_cnt[2 * BW + 2];
     __shared__ unsigned long long sm_red[BW];
-    extern __shared__ uint32_t dsm[];  // per warp: 32*(B+1) words
+    extern __shared__ uint32_t dsm[];  // per warp: 32*(B+1) words; then B*2K source hub values
     uint32_t* xs = dsm + (threadIdx.x >> 5) * 32 * (B + 1);
+    uint32_t* sh = dsm + BW * 32 * (B + 1);
     unsigned long long epoch = 0;
     const uint64_t tid = blockIdx.x * (uint64_t)BT + threadIdx.x;
     const uint64_t nthreads = (uint64_t)gridDim.x * BT;
@@ -410,11 +599,20 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
                 red_or(P.bitmap + (d >> 5), 1u << (d & 31));
             }
         }
+        if (P.HB) {  // the sources' hub values (certificates), per block
+            for (uint32_t i = threadIdx.x; i < (uint32_t)nq * 2 * P.K; i += BT) {
+                const uint32_t b = i / (2 * P.K), k = i % (2 * P.K);
+                const uint32_t s = __ldg(P.srcs + q0 + b);
+                const uint32_t col = k < P.K ? k : P.KP + (k - P.K);
+                sh[i] = s < P.n ? __ldg(P.HB + (size_t)s * 2 * P.KP + col) : 0u;
+            }
+        }
         grid_sync(P.ctrl, epoch);
 
         int phase = P.two_phase ? 1 : 2;
         bool predicate = false;
         bool bits = true;  // the current frontier is in the bitmap (seeds set bits), else in M
+        bool pull = false; // this iteration is the NEXT-1 pull over uncertified vertices
         uint32_t iters = 0, n_edges = 0, n_upd = 0;  // (edge, query) pairs of the whole batch
         for (;;) {
             const GraphView& g = (phase == 1) ? P.C : P.G;
@@ -425,7 +623,8 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
                 z[0] = z[1] = 0ull;
             }
             const unsigned long long t_s0 = (P.trace && tid == 0) ? global_ns() : 0ull;
-            compact_b<KIND, B>(P, g, predicate, !bits, ctr + CT_LIST, ctr + CT_ACTIVE, sm_cnt);
+            const int mode = pull ? F_UNCERT : predicate ? F_IMPACTED : bits ? F_BITS : F_MASKS;
+            compact_b<KIND, B>(P, pull ? P.R : g, mode, sh, nq, ctr + CT_LIST, ctr + CT_ACTIVE, sm_cnt);
             grid_sync(P.ctrl, epoch);
             ++ring;
             const unsigned long long ce = ld_cg64(ctr + CT_LIST);
@@ -444,6 +643,10 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
                 for (int b = 0; b < nq; ++b)  // union frontier, reported for every query of the batch
                     atomicAdd(P.stats + (size_t)(q0 + b) * NSTAT + (phase == 1 ? ST_F1 : ST_F2), a);
             }
+            if (E == 0 && pull) {  // nothing uncertified has an in-edge: phase 2 is already final
+                pull = false;
+                bits = false;
+            }
             if (E == 0) {
                 if (P.stats) {  // batch totals, attributed evenly to the batch's queries
                     block_add_split(P.stats, q0, nq, phase == 1 ? ST_E1 : ST_E2, n_edges, sm_red);
@@ -453,6 +656,7 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
                                   (unsigned long long)iters);
                 }
                 n_edges = n_upd = 0;
+                iters = 0;
                 if (phase == 1) {
                     if (P.p1) transpose_out<B>(P, P.p1, q0, nq, xs);
                     if (P.stats) {  // impacted per query (Alg 3 l.15); stride is a multiple of B: q fixed
@@ -461,10 +665,20 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
                         per_query_add<B>(P.stats, q0, nq, ST_IMP, c);
                     }
                     phase = 2;
-                    predicate = true;
+                    if (P.reduced) pull = true;   // Reduced(E): pull into uncertified vertices
+                    else predicate = true;        // Active <- impacted vertices (l.15)
                     continue;
                 }
                 break;
+            }
+            if (pull) {  // NEXT-1: one pull sweep, then push from the vertices it changed (masks in M)
+                relax_pull<KIND, PACKED, B>(P, count, E, xs, n_edges, n_upd);
+                pull = false;
+                bits = false;
+                grid_sync(P.ctrl, epoch);
+                if (P.trace && tid == 0 && tr < P.trace_cap) P.trace[5ull * tr + 2] = global_ns();
+                ++iters;
+                continue;
             }
             // small frontier: its S2 sets frontier bits (few reds) and the next S1 reads the bitmap;
             // large frontier: no bitmap reds (they contend in L2), the next S1 scans M instead
@@ -500,7 +714,7 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
 
 template <int KIND, bool PACKED, int B>
 void launch_b(const BParams& P, int sms, cudaStream_t s) {
-    const size_t smem = (size_t)BW * 32 * (B + 1) * sizeof(uint32_t);
+    const size_t smem = ((size_t)BW * 32 * (B + 1) + (size_t)B * 2 * 64) * sizeof(uint32_t);
     static int bps = 0;
     if (!bps) {
         if (smem > 48 * 1024)
@@ -560,6 +774,22 @@ void run_queries_batched(Graph& G, const QueryCall& c, int B, cudaStream_t s, st
     P.dmask = G.dbits >= 32 ? 0xffffffffu : ((1u << G.dbits) - 1u);
     P.G = view(*c.full_adj);
     P.C = c.two_phase ? view(*c.core_adj) : P.G;
+    P.R = view(G.gr);
+    {   // NEXT-1 (Reduced(E) pull) after phase 1 for the kinds with a certificate; CG_REDUCED is a
+        // bitmask over cg_kind.  Default REACH only: its certificate (reached = final) leaves only
+        // unreachable vertices; the SSWP / SSNP / SSSP certificates are exact but, united over a
+        // 16-query batch, leave ~99 % of the vertices uncertified for some query (measured, C2).
+        const char* e = getenv("CG_REDUCED");
+        const unsigned mask = e ? (unsigned)strtoul(e, nullptr, 0) : (1u << CG_REACH);
+        const Core& core = G.core[core_slot(c.kind)];
+        const bool has_cert = c.kind == CG_REACH || (core.hub_k > 0 && core.hub_k <= 64 && core.hub_vals.get());
+        P.reduced = c.two_phase && c.core_adj == &core.adj && ((mask >> c.kind) & 1u) && has_cert;
+        if (P.reduced && c.kind != CG_REACH) {
+            P.HB = core.hub_vals.get();
+            P.K = core.hub_k;
+            P.KP = (core.hub_k + 3) & ~3u;
+        }
+    }
     P.srcs = c.srcs;
     P.n_src = c.n_src;
     P.two_phase = c.two_phase;

@@ -39,6 +39,10 @@ struct Core {
     DevBuf<uint8_t> flags; // E_c membership in G's CSR edge order
     std::vector<uint32_t> hubs;
     float build_ms = 0.f;
+    // NEXT-1 certificates (Theorem 1 P:1321-1371 and its bottleneck analogs): the Identify
+    // queries' values kept as rows hub_vals[v][0..2K) = (Q(h_k) on G at v | Q(h_k) on G^R at v)
+    DevBuf<uint32_t> hub_vals;
+    uint32_t hub_k = 0;
 };
 
 struct Workspace {

@@ -14,7 +14,7 @@ from . import _lib
 KINDS = {"sssp": 0, "sswp": 1, "ssnp": 2, "viterbi": 3, "bfs": 4, "reach": 5}
 MODES = {"2phase": 0, "full": 1}
 HUB_POLICIES = {"topdeg": 0, "sampled": 1, "given": 2}
-CG_ALGS = {"auto": 0, "specialized": 1, "general": 2}
+CG_ALGS = {"auto": 0, "specialized": 1, "general": 2, "general_perdir": 3}
 
 
 def kind_id(kind) -> int:

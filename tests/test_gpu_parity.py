@@ -283,3 +283,36 @@ def test_batched_frontier_modes(bits_below, monkeypatch):
             out = to_np(g.query(kind, to_dev(sources), mode=mode))
             for i, s in enumerate(sources):
                 assert_values_equal(out[i], oracle.query(kind, og, int(s)), kind, f"bits<{bits_below} {kind} {mode}")
+
+
+@pytest.mark.parametrize("reduced", ["0", "0x3f"])
+def test_reduced_pull_completion(reduced, monkeypatch):
+    """NEXT-1: phase 2 = one pull sweep over the in-edges of vertices whose phase-1 value is not
+    certified (Theorem 1 P:1321-1371 and its bottleneck analogs; REACH: the lattice top), then
+    push.  Off (0) and on for every kind that has a certificate (0x3f): identical to the oracle."""
+    monkeypatch.setenv("CG_REDUCED", reduced)
+    n, m = 1 << 15, 16 << 15
+    src, dst, w = gen.rmat(n, m, w_max=9, seed=44)
+    g, og = both(n, src, dst, w)
+    sources = np.concatenate([[0], gen.sample_sources(n, src, dst, 21, seed=6)]).astype(np.uint32)
+    for kind in KINDS:
+        g.build(kind, K=20)
+        out = to_np(g.query(kind, to_dev(sources), mode="2phase"))
+        for i, s in enumerate(sources):
+            assert_values_equal(out[i], oracle.query(kind, og, int(s)), kind, f"reduced={reduced} {kind} s={s}")
+
+
+def test_general_cg_per_direction():
+    """Reading Q9 option: Alg 2 with one Qid[] per traversal direction == the oracle's option."""
+    n, m = 1 << 13, 12 << 13
+    src, dst, w = gen.rmat(n, m, seed=17)
+    g, og = both(n, src, dst, w)
+    ogr = oracle.transpose(og)
+    hubs = oracle.hubs_topdeg(og, ogr, 12)
+    g.build("reach", K=12, alg="general_perdir")
+    assert np.array_equal(g.core_flags("reach").cpu().numpy(), oracle.cg_alg2(og, ogr, hubs, per_direction=True))
+    s = gen.sample_sources(n, src, dst, 9, seed=3)
+    for kind in ("reach", "bfs"):
+        out = to_np(g.query(kind, to_dev(s), mode="2phase"))
+        for i, x in enumerate(s):
+            assert_values_equal(out[i], oracle.query(kind, og, int(x)), kind, "perdir")
