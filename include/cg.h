@@ -82,6 +82,9 @@ typedef struct {
     int64_t reached;                 /* |{v != s : Val(v) != InitVal}| after the query */
     int64_t precise_p1;              /* |{v != s reached : p1(v) == final(v)}| (Table 5, reading Q16);
                                         -1 unless the query kept phase-1 values */
+    int64_t scanned_p1, scanned_p2;  /* edge words the kernel read (pull sweep: in-edges).  Single-query
+                                        engine: == edges_*.  Batched: the union frontier's edges, each
+                                        read once for all queries of the batch, split evenly over them */
 } cg_stats;
 
 typedef void* (*cg_alloc_fn)(size_t bytes, void* stream, void* ctx);

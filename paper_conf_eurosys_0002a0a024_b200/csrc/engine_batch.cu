@@ -27,7 +27,7 @@ using namespace kern;
 constexpr int BT = 512;          // threads per CTA
 constexpr int BW = BT / 32;      // warps per CTA
 
-enum { ST_IT1, ST_IT2, ST_E1, ST_E2, ST_U1, ST_U2, ST_F1, ST_F2, ST_IMP, ST_REACH, ST_PREC, NSTAT };
+enum { ST_IT1, ST_IT2, ST_E1, ST_E2, ST_U1, ST_U2, ST_F1, ST_F2, ST_IMP, ST_REACH, ST_PREC, ST_S1, ST_S2, NSTAT };
 enum { CT0 = 8, CTS = 2, CT_LIST = 0, CT_ACTIVE = 1 };
 
 struct BParams {
@@ -614,6 +614,7 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
         bool bits = true;  // the current frontier is in the bitmap (seeds set bits), else in M
         bool pull = false; // this iteration is the NEXT-1 pull over uncertified vertices
         uint32_t iters = 0, n_edges = 0, n_upd = 0;  // (edge, query) pairs of the whole batch
+        unsigned long long n_scan = 0;                // union edges read (every thread keeps the sum)
         for (;;) {
             const GraphView& g = (phase == 1) ? P.C : P.G;
             const int slot = ring & 3;
@@ -647,7 +648,13 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
                 pull = false;
                 bits = false;
             }
+            n_scan += E;
             if (E == 0) {
+                if (P.stats && tid == 0 && n_scan)
+                    for (int b = 0; b < nq; ++b)
+                        atomicAdd(P.stats + (size_t)(q0 + b) * NSTAT + (phase == 1 ? ST_S1 : ST_S2),
+                                  n_scan / nq + (b == 0 ? n_scan % nq : 0));
+                n_scan = 0;
                 if (P.stats) {  // batch totals, attributed evenly to the batch's queries
                     block_add_split(P.stats, q0, nq, phase == 1 ? ST_E1 : ST_E2, n_edges, sm_red);
                     block_add_split(P.stats, q0, nq, phase == 1 ? ST_U1 : ST_U2, n_upd, sm_red);
@@ -869,6 +876,8 @@ void run_queries_batched(Graph& G, const QueryCall& c, int B, cudaStream_t s, st
             o.impacted = (int64_t)x[ST_IMP];
             o.reached = (int64_t)x[ST_REACH];
             o.precise_p1 = P.p1 ? (int64_t)x[ST_PREC] : -1;
+            o.scanned_p1 = (int64_t)x[ST_S1];
+            o.scanned_p2 = (int64_t)x[ST_S2];
         }
     }
 }
