@@ -43,7 +43,7 @@ def parse():
     p.add_argument("--steps", type=int, default=10)
     p.add_argument("--warmup", type=int, default=3)
     p.add_argument("--config", default="c2")
-    p.add_argument("--batch", type=int, default=16, help="sources per kind per step (per GPU)")
+    p.add_argument("--batch", type=int, default=32, help="sources per kind per step (per GPU)")
     p.add_argument("--K", type=int, default=20, help="Core Graph hubs")
     p.add_argument("--kinds", default=",".join(KINDS))
     p.add_argument("--impl", default="native", choices=["native", "reference"])
@@ -325,7 +325,6 @@ def main():
     # ---- per-query counters (untimed): algorithmic bytes, EDGES-RED, p1 precision
     per_kind = {}
     alg_bytes_2p = {}
-    bw = int(os.environ.get("CG_BATCH", "16"))  # the library's batch width (engine_batch.cu batch_width)
     eb = 4 if (int(cfg.n - 1).bit_length() + int(cfg.w_max - 1).bit_length()) <= 32 else 8  # packed edge word?
     for k in kinds:
         _, p1, st2 = g.query(k, srcs[k], mode="2phase", p1=True, stats=True)
@@ -337,20 +336,22 @@ def main():
         precise = sum(s["precise_p1"] for s in st2)
 
         def bytes_of(sts, two_phase):
-            # algorithmic bytes of the batched query kernel: per launch of Bw-wide
-            # batches — value rows initialised (4 n Bw) and masks cleared (4 n); per union-frontier
-            # vertex 2x4 B row offsets + its 4 Bw B value row + 3x4 B list entry written and read;
-            # per union edge one edge word (4 B packed / 8 B wide) + v's 4 Bw B value row; per
-            # EdgeFunction a 4 B atomic; the impacted scan (2Phase, 4 n Bw); the transpose out
-            # (4 n Bw read + 4 n per query written)
-            tot = 0
-            for q0 in range(0, len(sts), bw):
-                grp = sts[q0:q0 + bw]
+            # algorithmic bytes of the batched query kernel, per pass of Qb queries
+            # with RB-byte value rows (cg_stats.batch_queries / row_bytes): rows initialised
+            # (n RB) and masks cleared (4 n); per union-frontier vertex 8 B of row offsets + its
+            # RB row + 3x4 B list entry written and read; per union edge one edge word (4 B packed
+            # / 8 B wide) + v's RB row; per EdgeFunction a 4 B atomic; the impacted scan (2Phase,
+            # n RB); the transpose out (n RB read + 4 n per query written)
+            tot, i = 0, 0
+            while i < len(sts):
+                qb, rb = max(1, sts[i]["batch_queries"]), sts[i]["row_bytes"]
+                grp = sts[i:i + qb]
+                i += qb
                 fr = grp[0]["frontier_p1"] + grp[0]["frontier_p2"]  # union frontier (same for the batch)
                 sc = sum(s["scanned_p1"] + s["scanned_p2"] for s in grp)
                 up = sum(s["updates_p1"] + s["updates_p2"] for s in grp)
-                tot += 4 * cfg.n * bw + 4 * cfg.n + fr * (8 + 4 * bw + 24) + sc * (eb + 4 * bw) + 4 * up
-                tot += (4 * cfg.n * bw if two_phase else 0) + 4 * cfg.n * bw + 4 * cfg.n * len(grp)
+                tot += cfg.n * rb + 4 * cfg.n + fr * (8 + rb + 24) + sc * (eb + rb) + 4 * up
+                tot += (cfg.n * rb if two_phase else 0) + cfg.n * rb + 4 * cfg.n * len(grp)
             return tot
         alg_bytes_2p[k] = bytes_of(st2, True)
         mean2 = statistics.mean(kms2[k])
@@ -378,7 +379,7 @@ def main():
     # per-query figure (profiles/ncu_query_kernel.json); None when no capture exists
     traffic = tr["dram_bytes_per_query"] * B if tr else None
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                "traffic": traffic, "kernel": "batch_kernel<KIND,packed,16> (one launch per kind per step)",
+                "traffic": traffic, "kernel": "batch_kernel<KIND,packed,lanes> (one launch per kind per step)",
                 "peak_source": peak_src,
                 "alg_bytes_per_launch": tot_bytes / len(kinds)}
 

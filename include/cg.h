@@ -85,6 +85,9 @@ typedef struct {
     int64_t scanned_p1, scanned_p2;  /* edge words the kernel read (pull sweep: in-edges).  Single-query
                                         engine: == edges_*.  Batched: the union frontier's edges, each
                                         read once for all queries of the batch, split evenly over them */
+    int32_t batch_queries;           /* queries per pass of the engine that ran this query (1: single-query) */
+    int32_t row_bytes;               /* bytes of one vertex's value row in that pass (u32 lanes: 4 per query;
+                                        u8 lanes: 1 per query; REACH bit lanes: 1 bit per query) */
 } cg_stats;
 
 typedef void* (*cg_alloc_fn)(size_t bytes, void* stream, void* ctx);

@@ -49,7 +49,8 @@ class Stats(ctypes.Structure):
                 ("frontier_p1", ctypes.c_int64), ("frontier_p2", ctypes.c_int64),
                 ("impacted", ctypes.c_int64), ("reached", ctypes.c_int64),
                 ("precise_p1", ctypes.c_int64),
-                ("scanned_p1", ctypes.c_int64), ("scanned_p2", ctypes.c_int64)]
+                ("scanned_p1", ctypes.c_int64), ("scanned_p2", ctypes.c_int64),
+                ("batch_queries", ctypes.c_int32), ("row_bytes", ctypes.c_int32)]
 
     def as_dict(self) -> dict:
         return {k: int(getattr(self, k)) for k, _ in self._fields_}

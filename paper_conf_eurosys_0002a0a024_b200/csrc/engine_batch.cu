@@ -1,22 +1,27 @@
-// engine_batch.cu — SURVEY §8(f) NEXT-2: batched multi-source relaxation.  B independent
+// engine_batch.cu — SURVEY §8(f) NEXT-2: batched multi-source relaxation.  Q independent
 // queries of one kind (vertex queries are independent) run through Alg 3
 // in lock-step on one persistent kernel:
 //
-//   * values live as V[v][q] (a 32·B-byte row per vertex), so ONE gather of v's row serves the
-//     Needed test of all B queries: the random-access cost that bounds the single-query sweep
-//     (one 32 B sector per edge per query) drops B-fold;
+//   * values live as a ROW per vertex holding all Q queries' values, so ONE gather of v's row
+//     serves the Needed test of every query: the random-access cost that bounds the
+//     single-query sweep (one 32 B sector per edge per query) is shared by the batch;
+//   * rows are packed by value lanes (Lanes32 / Lanes16 / LanesBit below): u32 lanes (the
+//     Table 6 types; Viterbi, and the fallback of every kind) with Q = 16 — a 64 B row; binary16
+//     lanes (SSSP / SSWP / SSNP / BFS: small integers, exact) with Q = 32 — a 64 B row; one bit
+//     per query (REACH) with Q = 32 — a 4 B row.  The EdgeFunction of 8 binary16 lanes is one
+//     vector red.min/max (REDG.F16x8), of 32 bit lanes one red.or;
 //   * the frontier is the union over the batch: a vertex bitmap plus a per-vertex mask M[v]
 //     of the queries for which v is active; phase 1 / phase 2 switch when the union converges;
-//   * a lane handles one edge for all B queries: one edge word, one vector load of v's row,
-//     u's row from shared memory, B Needed tests, red.min/max only for the needed queries;
-//   * the same S1 / S2 structure as engine.cu (CTA-aggregated compaction, edge-balanced split
-//     of the union frontier's edges over all warps, red.min / red.max EdgeFunction);
-//   * finally the batch is transposed into the caller's [query][vertex] layout.
+//   * S1 / S2 as in engine.cu: CTA-aggregated compaction into an edge-offset list, the
+//     iteration's edges split evenly over all warps; a lane takes one edge for all Q queries,
+//     its value row copied global -> shared (cp.async) one 32-edge chunk ahead;
+//   * finally the batch is transposed into the caller's [query][vertex] u32 layout.
 #include <cstdio>
 #include <cstdlib>
 
-#include "kernels.cuh"
+#include <cuda_fp16.h>
 
+#include "kernels.cuh"
 
 namespace cgb {
 
@@ -26,9 +31,14 @@ using namespace kern;
 
 constexpr int BT = 512;          // threads per CTA
 constexpr int BW = BT / 32;      // warps per CTA
+#ifndef CGB_STAGES
+#define CGB_STAGES 2
+#endif
+constexpr int S_PIPE = CGB_STAGES;  // value-row pipeline depth (chunks of 32 edges per warp)
 
 enum { ST_IT1, ST_IT2, ST_E1, ST_E2, ST_U1, ST_U2, ST_F1, ST_F2, ST_IMP, ST_REACH, ST_PREC, ST_S1, ST_S2, NSTAT };
 enum { CT0 = 8, CTS = 2, CT_LIST = 0, CT_ACTIVE = 1 };
+enum { ERR_ITERS = 1u, ERR_SOURCE = 2u, ERR_LANE_OVERFLOW = 4u };
 
 struct BParams {
     uint32_t n, words, dbits, dmask;
@@ -38,7 +48,7 @@ struct BParams {
     int two_phase;
     uint32_t* out;              // caller layout: out[q * n + v]
     uint32_t* p1;               // nullable, caller layout
-    uint32_t* V;                // [n][B] batch values
+    uint32_t* V;                // [n][RW] value rows
     uint32_t* M;                // [n] active-query masks
     uint32_t* bitmap;           // [words] union frontier
     uint32_t* lv;               // compacted union frontier: vertex, edge offset, query mask
@@ -50,7 +60,7 @@ struct BParams {
     uint32_t max_iters;
     uint32_t bits_below;        // frontiers smaller than this keep a bitmap (else the masks M are scanned)
     GraphView R;                // G^R: in-edges for the NEXT-1 pull
-    const uint32_t* HB;         // CG hub rows [n][2K] for the certificates (nullable)
+    const uint32_t* HB;         // CG hub rows [n][2K] for the certificates (nullable; u32 lanes only)
     uint32_t K, KP;             // hubs in HB; row stride 2*KP (KP = K rounded up to a multiple of 4)
     int reduced;                // phase 2 starts with the certificate-driven pull (NEXT-1)
     uint32_t fresh;             // bit p-1: phase p pre-reads values from L2 instead of L1
@@ -58,19 +68,147 @@ struct BParams {
     uint32_t trace_cap;
 };
 
-// does row v hold a non-InitVal value for any query (and which)?
-template <int KIND, int B>
-__device__ __forceinline__ uint32_t row_mask(const uint32_t* V, uint32_t v) {
+// ------------------------------------------------------------------ value lanes
+// A row = RW u32 words = Q query lanes, QPW lanes per word.  Per policy:
+//   init_word()          every lane InitVal (Alg 3 l.4, l.6)
+//   decode(word, j)      lane j in the caller's u32 encoding (Table 6 values; binary32 for Viterbi)
+//   live(word)           QPW-bit mask of lanes != InitVal (reached)
+//   top(word)            QPW-bit mask of lanes == the lattice top (final by definition)
+//   seed(p, j, val)      set lane j of *p (a word holding InitVal there) to the encoded val
+//   src_val(), nb_val(w) SourceInitVal and SourceInitVal (+) w, encoded (Alg 3 l.5, l.8)
+//   relax(p, uw, cw, w, act, ...)  Process + EdgeFunction of one word (Alg 3 l.22-27): the lanes
+//       of act whose candidate ext(uw, w) is better than cw; returns the changed lanes
+template <int KIND>
+struct Lanes32 {  // one u32 per query (Table 6 types)
     using O = Op<KIND>;
-    uint32_t m = 0;
-    const uint4* r = reinterpret_cast<const uint4*>(V + (size_t)v * B);
-#pragma unroll
-    for (int i = 0; i < B / 4; ++i) {
-        uint4 x;
-        asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(x.x), "=r"(x.y), "=r"(x.z), "=r"(x.w) : "l"(r + i));
-        m |= (uint32_t)(x.x != O::INIT) << (4 * i) | (uint32_t)(x.y != O::INIT) << (4 * i + 1) |
-             (uint32_t)(x.z != O::INIT) << (4 * i + 2) | (uint32_t)(x.w != O::INIT) << (4 * i + 3);
+    static constexpr int Q = 16, QPW = 1, RW = 16, G = 1;
+    __device__ static uint32_t init_word() { return O::INIT; }
+    __device__ static uint32_t decode(uint32_t x, uint32_t) { return x; }
+    __device__ static uint32_t live(uint32_t x) { return x != O::INIT; }
+    __device__ static uint32_t top(uint32_t x) { return x == O::SRC; }
+    __device__ static void seed(uint32_t* p, uint32_t, uint32_t val) { *p = val; }
+    __device__ static uint32_t src_val() { return O::SRC; }
+    __device__ static uint32_t nb_val(uint32_t w) { return O::ext(O::SRC, w); }
+    __device__ static uint32_t relax(uint32_t* p, const uint32_t (&u)[G], const uint32_t (&c)[G], uint32_t w,
+                                     uint32_t act, uint32_t& n_edges, uint32_t& n_upd, uint32_t*) {
+        if (!act || u[0] == O::INIT) return 0u;  // (a pull may read an unreached u)
+        ++n_edges;
+        const uint32_t cand = O::ext(u[0], w);
+        if (!O::better(cand, c[0])) return 0u;  // Needed(e(u,v))
+        O::edge_fn(p, cand);                  // EdgeFunction
+        ++n_upd;
+        return 1u;
     }
+};
+
+// f16 lanes (binary16 numbers; their bit patterns order like the values because all values
+// are >= 0): SSSP / SSNP / BFS: InitVal +inf, SourceInitVal 0, select min; SSWP: InitVal 0,
+// SourceInitVal +inf (above every weight), select max.  Integers up to 2048 are exact in
+// binary16: SSWP / SSNP values are edge weights (the host requires w_max <= 2048); SSSP / BFS
+// raise ERR_LANE_OVERFLOW when a candidate reaches 2048 and the host re-runs the call with u32
+// lanes.  The EdgeFunction of 8 lanes is ONE red.min/max.noftz.v4.f16x2 (REDG.F16x8) of a
+// 16 B chunk whose non-improving lanes hold the neutral value.  Decoded +inf is 0xFFFFFFFF (SSWP's
+// SourceInitVal, the other kinds' InitVal).
+template <int KIND>
+struct Lanes16 {
+    static_assert(KIND == CG_SSSP || KIND == CG_SSWP || KIND == CG_SSNP || KIND == CG_BFS, "f16 lanes");
+    static constexpr int Q = 32, QPW = 2, RW = 16, G = 4;
+    static constexpr bool MAXK = KIND == CG_SSWP;
+    static constexpr uint32_t INF16 = 0x7c00u, LIMIT = 0x68006800u;  // +inf; 2048.0 in both lanes
+    static constexpr uint32_t INIT16 = MAXK ? 0u : INF16, SRC16 = MAXK ? INF16 : 0u;
+    __device__ static uint32_t init_word() { return INIT16 * 0x10001u; }
+    __device__ static uint32_t decode(uint32_t x, uint32_t j) {
+        const uint32_t h = (x >> (16 * j)) & 0xffffu;
+        return h == INF16 ? 0xffffffffu : (uint32_t)__half2float(__ushort_as_half((unsigned short)h));
+    }
+    __device__ static uint32_t bits2(uint32_t m) { return ((m >> 15) & 1u) | ((m >> 30) & 2u); }  // 0xffff lanes -> 2 bits
+    __device__ static uint32_t halves2(uint32_t b) { return ((b & 1u) ? 0xffffu : 0u) | ((b & 2u) ? 0xffff0000u : 0u); }
+    __device__ static uint32_t live(uint32_t x) { return bits2(__vcmpne2(x, init_word())); }
+    __device__ static uint32_t top(uint32_t x) { return bits2(__vcmpeq2(x, SRC16 * 0x10001u)); }
+    __device__ static void seed(uint32_t* p, uint32_t j, uint32_t val) {  // one writer per (vertex, lane)
+        reinterpret_cast<unsigned short*>(p)[j] = (unsigned short)val;
+    }
+    __device__ static uint32_t src_val() { return SRC16; }
+    __device__ static uint32_t h16(uint32_t w) { return __half_as_ushort(__uint2half_rn(w)); }
+    __device__ static uint32_t nb_val(uint32_t w) { return KIND == CG_BFS ? 0x3c00u : h16(w); }
+    __device__ static uint32_t ext2(uint32_t u, uint32_t w2) {
+        const __half2 a = *reinterpret_cast<const __half2*>(&u), b = *reinterpret_cast<const __half2*>(&w2);
+        __half2 r;
+        if (KIND == CG_SSWP) r = __hmin2(a, b);
+        else if (KIND == CG_SSNP) r = __hmax2(a, b);
+        else r = __hadd2(a, b);  // SSSP: + w; BFS: + 1
+        return *reinterpret_cast<const uint32_t*>(&r);
+    }
+    // Process + EdgeFunction of one 16 B chunk (4 words, 8 queries); act: 8 query bits
+    __device__ static uint32_t relax(uint32_t* p, const uint32_t (&u)[G], const uint32_t (&c)[G], uint32_t w,
+                                     uint32_t act, uint32_t& n_edges, uint32_t& n_upd, uint32_t* err) {
+        if (!act) return 0u;
+        n_edges += __popc(act);
+        const uint32_t w2 = (KIND == CG_BFS ? 0x3c00u : h16(w)) * 0x10001u;
+        uint32_t cand[G], ch = 0, over = 0;
+#pragma unroll
+        for (int i = 0; i < G; ++i) {
+            const uint32_t am = halves2(act >> (2 * i));
+            const uint32_t x = ext2(u[i], w2);
+            const uint32_t bm = (MAXK ? __vcmpgtu2(x, c[i]) : __vcmpltu2(x, c[i])) & am;  // Needed, 2 queries
+            if (KIND == CG_SSSP || KIND == CG_BFS) over |= __vcmpgeu2(x, LIMIT) & bm;
+            cand[i] = MAXK ? (x & bm) : ((x & bm) | (INF16 * 0x10001u & ~bm));  // others neutral
+            ch |= bits2(bm) << (2 * i);
+        }
+        if (over) atomicOr(err, ERR_LANE_OVERFLOW);
+        if (!ch) return 0u;
+        if (MAXK)
+            asm volatile("red.relaxed.gpu.global.max.noftz.v4.f16x2 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(cand[0]),
+                         "r"(cand[1]), "r"(cand[2]), "r"(cand[3])
+                         : "memory");
+        else
+            asm volatile("red.relaxed.gpu.global.min.noftz.v4.f16x2 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(cand[0]),
+                         "r"(cand[1]), "r"(cand[2]), "r"(cand[3])
+                         : "memory");
+        n_upd += __popc(ch);
+        return ch;
+    }
+};
+
+// one bit per query (REACH): InitVal 0, SourceInitVal 1, cand = u; EdgeFunction red.or
+struct LanesBit {
+    static constexpr int Q = 32, QPW = 32, RW = 1, G = 1;
+    __device__ static uint32_t init_word() { return 0u; }
+    __device__ static uint32_t decode(uint32_t x, uint32_t j) { return (x >> j) & 1u; }
+    __device__ static uint32_t live(uint32_t x) { return x; }
+    __device__ static uint32_t top(uint32_t x) { return x; }
+    __device__ static void seed(uint32_t* p, uint32_t j, uint32_t) { atomicOr(p, 1u << j); }
+    __device__ static uint32_t src_val() { return 1u; }
+    __device__ static uint32_t nb_val(uint32_t) { return 1u; }
+    __device__ static uint32_t relax(uint32_t* p, const uint32_t (&u)[G], const uint32_t (&c)[G], uint32_t,
+                                     uint32_t act, uint32_t& n_edges, uint32_t& n_upd, uint32_t*) {
+        n_edges += __popc(act);
+        const uint32_t nw = u[0] & act & ~c[0];  // Needed: u reached, v not
+        if (!nw) return 0u;
+        red_or(p, nw);
+        n_upd += __popc(nw);
+        return nw;
+    }
+};
+
+template <int LW, int KIND> struct LanesOf;
+template <int KIND> struct LanesOf<32, KIND> { using T = Lanes32<KIND>; };
+template <int KIND> struct LanesOf<16, KIND> { using T = Lanes16<KIND>; };
+template <int KIND> struct LanesOf<1, KIND> { using T = LanesBit; };
+
+template <class L>
+__device__ __forceinline__ uint32_t group_mask(uint32_t mask, int i) {  // the lanes of word group i in a query mask
+    constexpr int LG = L::QPW * L::G;  // lanes per relax group
+    return LG >= 32 ? mask : (mask >> (i * LG)) & ((1u << LG) - 1u);
+}
+
+// queries with a non-InitVal value at v (L2 reads: values other SMs update)
+template <class L>
+__device__ __forceinline__ uint32_t row_live(const uint32_t* V, uint32_t v) {
+    const uint32_t* r = V + (size_t)v * L::RW;
+    uint32_t m = 0;
+#pragma unroll
+    for (int i = 0; i < L::RW; ++i) m |= L::live(ld_cg(r + i)) << (i * L::QPW);
     return m;
 }
 
@@ -94,25 +232,18 @@ __device__ __forceinline__ bool certified(uint32_t p, uint32_t Fv, uint32_t Rv, 
     return false;
 }
 
-// queries q < nq whose phase-1 value at v is not proven final (Reduced(E) keeps v's in-edges).
-// Kept register-light (it runs inside the persistent kernel): the value row is only compared,
-// then each open query re-reads its value and scans the hub row 4 hubs per 16 B load.
-template <int KIND, int B>
+// queries q < nq whose phase-1 value at v is not proven final (Reduced(E) keeps v's in-edges):
+// the lattice top is final (REACH: reached); u32 lanes may add the hub certificates.  Kept
+// register-light (it runs inside the persistent kernel).
+template <int KIND, class L>
 __device__ uint32_t uncertified(const BParams& P, const uint32_t* sh, int nq, uint32_t v) {
-    using O = Op<KIND>;
-    const uint32_t* row = P.V + (size_t)v * B;
+    constexpr uint32_t WM = L::QPW == 32 ? 0xffffffffu : (1u << L::QPW) - 1u;
+    const uint32_t* row = P.V + (size_t)v * L::RW;
     uint32_t unc = 0;
 #pragma unroll
-    for (int i = 0; i < B / 4; ++i) {
-        uint4 x;
-        asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];"
-                     : "=r"(x.x), "=r"(x.y), "=r"(x.z), "=r"(x.w)
-                     : "l"(reinterpret_cast<const uint4*>(row) + i));
-        unc |= (uint32_t)(x.x != O::SRC) << (4 * i) | (uint32_t)(x.y != O::SRC) << (4 * i + 1) |
-               (uint32_t)(x.z != O::SRC) << (4 * i + 2) | (uint32_t)(x.w != O::SRC) << (4 * i + 3);
-    }
-    unc &= nq >= 32 ? 0xffffffffu : ((1u << nq) - 1u);  // the lattice top (REACH: reached) is final
-    if (KIND == CG_REACH || P.HB == nullptr || !unc) return unc;
+    for (int i = 0; i < L::RW; ++i) unc |= (~L::top(ld_cg(row + i)) & WM) << (i * L::QPW);
+    unc &= nq >= 32 ? 0xffffffffu : ((1u << nq) - 1u);
+    if (L::QPW != 1 || KIND == CG_REACH || P.HB == nullptr || !unc) return unc;
     // hub row of v: F at [0, KP), R at [KP, 2 KP) (KP = K rounded up to 4: 16 B aligned chunks)
     const uint32_t K = P.K, KP = P.KP;
     const uint4* hb = reinterpret_cast<const uint4*>(P.HB + (size_t)v * 2 * KP);
@@ -145,12 +276,14 @@ __device__ uint32_t uncertified(const BParams& P, const uint32_t* sh, int nq, ui
 // mode: F_BITS (frontier bits set by S2), F_MASKS (frontier = {v : M[v] != 0}), F_IMPACTED
 // (Alg 3 l.15: v active for q iff Val(v) != InitVal), F_UNCERT (NEXT-1: v active for its
 // uncertified queries; degrees are then in-degrees, g = G^R).
+// Pass 1 counts the active vertices with edges and their edges per warp and reserves the CTA's
+// list range with ONE 64-bit atomicAdd; pass 2 writes (v, edge offset, query mask) in vertex
+// order, consuming the masks and the bitmap bits.
 enum { F_BITS = 0, F_MASKS = 1, F_IMPACTED = 2, F_UNCERT = 3 };
 
-template <int KIND, int B>
-__device__ void compact_b(const BParams& P, const GraphView& g, int mode, const uint32_t* sh, int nq,
-                          unsigned long long* cnt_slot, unsigned long long* act_slot, uint32_t* sm) {
-    const bool predicate = mode == F_IMPACTED;
+template <int KIND, class L>
+__device__ void compact(const BParams& P, const GraphView& g, int mode, const uint32_t* sh, int nq,
+                        unsigned long long* cnt_slot, unsigned long long* act_slot, uint32_t* sm) {
     const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const uint64_t W = P.words;
     const uint32_t w0 = (uint32_t)(W * blockIdx.x / gridDim.x), w1 = (uint32_t)(W * (blockIdx.x + 1) / gridDim.x);
@@ -160,29 +293,33 @@ __device__ void compact_b(const BParams& P, const GraphView& g, int mode, const 
     for (uint32_t g0 = w0 + warp * 32; g0 < w1; g0 += BW * 32) {
         const uint32_t wi = g0 + lane;
         uint32_t word = 0;
-        if (predicate) {  // Alg 3 l.15 for every query of the batch: v active iff some Val(v) != InitVal
+        if (mode == F_IMPACTED) {  // Alg 3 l.15 for every query of the batch
             for (uint32_t j = 0; j < 32; ++j) {
                 const uint32_t v = (g0 + j) * 32 + lane;
-                const bool act = g0 + j < w1 && v < P.n && row_mask<KIND, B>(P.V, v) != 0;
+                const bool act = g0 + j < w1 && v < P.n && row_live<L>(P.V, v) != 0;
                 const uint32_t bits = __ballot_sync(FULL, act);
                 if (lane == j) word = bits;
             }
-            if (wi < w1 && word) P.bitmap[wi] = word;
+            if (wi < w1) P.bitmap[wi] = word;
         } else if (mode == F_UNCERT) {  // certificates: the uncertified queries' mask parks in M
             for (uint32_t j = 0; j < 32; ++j) {
                 const uint32_t v = (g0 + j) * 32 + lane;
-                const uint32_t unc = (g0 + j < w1 && v < P.n) ? uncertified<KIND, B>(P, sh, nq, v) : 0u;
+                const uint32_t unc = (g0 + j < w1 && v < P.n) ? uncertified<KIND, L>(P, sh, nq, v) : 0u;
                 if (unc) P.M[v] = unc;
                 const uint32_t bits = __ballot_sync(FULL, unc != 0);
                 if (lane == j) word = bits;
             }
             if (wi < w1) P.bitmap[wi] = word;
-        } else if (mode == F_MASKS) {  // union frontier = {v : M[v] != 0}: the last S2 set no bitmap bits
-#pragma unroll 8
+        } else if (mode == F_MASKS) {  // union frontier = {v : M[v] != 0}: all 32 loads in flight
+            uint32_t mv[32];
+#pragma unroll
             for (uint32_t j = 0; j < 32; ++j) {
                 const uint32_t v = (g0 + j) * 32 + lane;
-                const bool act = g0 + j < w1 && v < P.n && ld_cg(P.M + v) != 0u;
-                const uint32_t bits = __ballot_sync(FULL, act);
+                mv[j] = (g0 + j < w1 && v < P.n) ? ld_cg(P.M + v) : 0u;
+            }
+#pragma unroll
+            for (uint32_t j = 0; j < 32; ++j) {
+                const uint32_t bits = __ballot_sync(FULL, mv[j] != 0u);
                 if (lane == j) word = bits;
             }
             if (wi < w1) P.bitmap[wi] = word;
@@ -252,8 +389,8 @@ __device__ void compact_b(const BParams& P, const GraphView& g, int mode, const 
                 const uint32_t d = act ? deg[k] : 0u;
                 uint32_t mask = 0;
                 if (act) {
-                    if (predicate) {
-                        mask = row_mask<KIND, B>(P.V, v);
+                    if (mode == F_IMPACTED) {
+                        mask = row_live<L>(P.V, v);
                     } else {
                         mask = ld_cg(P.M + v);
                         P.M[v] = 0u;  // consumed
@@ -279,55 +416,145 @@ __device__ void compact_b(const BParams& P, const GraphView& g, int mode, const 
     }
 }
 
-// ------------------------------------------------------------------ S2 (lane = edge, vector over queries)
-// Same edge-balanced split and 32-row windows as engine.cu; a lane handles one edge for all B
-// queries: one edge word, one B-value row of v (vector loads), the row of u from shared memory.
-template <int B>
-struct Row {
-    uint32_t x[B];
-    // Needed pre-read of all B values: L1-allocating (may be stale, never better), or from L2
-    // (fresher: fewer redundant EdgeFunction atomics where values still change a lot)
-    __device__ void load(const uint32_t* p, bool fresh) {
-#pragma unroll
-        for (int i = 0; i < B / 4; ++i) {
-            uint4 t;
-            if (fresh)
-                asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];"
-                             : "=r"(t.x), "=r"(t.y), "=r"(t.z), "=r"(t.w)
-                             : "l"(p + 4 * i));
-            else
-                asm volatile("ld.global.ca.v4.u32 {%0,%1,%2,%3}, [%4];"
-                             : "=r"(t.x), "=r"(t.y), "=r"(t.z), "=r"(t.w)
-                             : "l"(p + 4 * i));
-            x[4 * i] = t.x;
-            x[4 * i + 1] = t.y;
-            x[4 * i + 2] = t.z;
-            x[4 * i + 3] = t.w;
-        }
-    }
-    __device__ void load_smem(const uint32_t* p) {
-#pragma unroll
-        for (int i = 0; i < B / 4; ++i) {
-            const uint4 t = reinterpret_cast<const uint4*>(p)[i];
-            x[4 * i] = t.x;
-            x[4 * i + 1] = t.y;
-            x[4 * i + 2] = t.z;
-            x[4 * i + 3] = t.w;
+// ------------------------------------------------------------------ S2 (lane = edge, row over queries)
+// Bytes of one (<= 16 B) cp.async copy of a row, copies per row, and the XOR swizzle of a lane's
+// row in a pipeline stage: copy i of lane L's row sits at slot i ^ sw(L), so the 32 lanes'
+// shared-memory reads of word w hit all banks.
+template <class L> struct RowCopy {
+    static constexpr uint32_t CB = L::RW >= 4 ? 16u : 4u * L::RW;  // bytes per copy
+    static constexpr uint32_t CW4 = CB / 4;                         // words per copy
+    static constexpr uint32_t C = L::RW / CW4;                      // copies per row
+    static constexpr uint32_t LPL = 4 * L::RW >= 128 ? 1u : 128u / (4 * L::RW);  // lanes per 128 B
+    __device__ static uint32_t sw(uint32_t lane) { return C > 1 ? (lane / LPL) % C : 0u; }
+    __device__ static void copy(uint32_t* dst, const uint32_t* src, bool fresh) {
+        if (CB == 16) {
+            if (fresh) cp_async16_cg(dst, src);  // Needed pre-read from L2
+            else cp_async16_ca(dst, src);        // from L1 (a stale value is never better)
+        } else {
+            asm volatile("cp.async.ca.shared.global [%0], [%1], %2;" ::"r"(smem_u32(dst)), "l"(src), "n"(CB) : "memory");
         }
     }
 };
 
-template <int KIND, bool PACKED, int B>
-__device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, uint32_t E, uint32_t* xs /* 32*B */,
-                        bool set_bits, bool fresh, uint32_t& n_edges, uint32_t& n_upd) {
-    using O = Op<KIND>;
-    constexpr int U = 2;  // edges per lane in flight
+// The edges [e, ehi) of one 32-row window: lane r of the window holds row r's first edge index
+// `off`, its address base (edge address = base + edge index) and its query mask; the rows'
+// values are in xs (r * RW + word).  Lane L takes edge L of each 32-edge chunk for all Q queries.
+// Software pipeline (S_PIPE stages, per-warp ring `vs` in shared memory): the edge word of chunk
+// c + S is loaded when chunk c + S - 1's value rows are requested (cp.async global -> shared),
+// while chunk c is consumed.
+template <int KIND, bool PACKED, class L>
+__device__ __forceinline__ void window_edges(const BParams& P, const GraphView& g, const uint32_t* xs, uint32_t* vs,
+                                             uint32_t off, uint32_t base, uint32_t mask, uint32_t e, uint32_t ehi,
+                                             bool set_bits, bool fresh, uint32_t& n_edges, uint32_t& n_upd,
+                                             uint32_t& n_read) {
+    constexpr int S = S_PIPE, RW = L::RW;
+    using RC = RowCopy<L>;
+    constexpr uint32_t NONE = 0xffffffffu;
     const uint32_t lane = threadIdx.x & 31;
-    const uint32_t gw = blockIdx.x * BW + (threadIdx.x >> 5);
-    const uint64_t NW = (uint64_t)gridDim.x * BW;
-    const uint32_t e0 = (uint32_t)((uint64_t)E * gw / NW), e1 = (uint32_t)((uint64_t)E * (gw + 1) / NW);
-    if (e0 >= e1) return;
+    const uint32_t swz = RC::sw(lane);
+    if (e >= ehi) return;
+    const uint32_t nch = (ehi - e + 31) >> 5;
 
+    EdgeWord<PACKED> ew[S];        // fetched edge words, chunk c + S ahead
+    uint32_t ek[S];                // their window row (NONE: no edge / inactive row)
+    uint32_t sd[S], sw[S], sk[S];  // requested chunks: destination, weight, window row
+
+    auto fetch = [&](uint32_t c, EdgeWord<PACKED>& wd, uint32_t& kout) {
+        const uint32_t t = e + c * 32 + lane;
+        uint32_t kk = 0;
+#pragma unroll
+        for (uint32_t st = 16; st > 0; st >>= 1)
+            if (__shfl_sync(FULL, off, kk + st) <= t) kk += st;
+        const uint32_t mk = __shfl_sync(FULL, mask, kk);
+        const uint32_t a = __shfl_sync(FULL, base, kk) + t;
+        const bool ok = t < ehi && mk != 0u;
+        if (ok) wd.load(g, a);
+        kout = ok ? kk : NONE;
+    };
+    auto request = [&](int slot, const EdgeWord<PACKED>& wd, uint32_t kk) {
+        sk[slot] = kk;
+        if (kk != NONE) {
+            uint32_t d, w;
+            wd.decode(P.dbits, P.dmask, d, w);
+            sd[slot] = d;
+            sw[slot] = w;
+            const uint32_t* src = P.V + (size_t)d * RW;
+            uint32_t* dst = vs + (slot * 32 + lane) * RW;
+#pragma unroll
+            for (uint32_t i = 0; i < RC::C; ++i) RC::copy(dst + RC::CW4 * (i ^ swz), src + RC::CW4 * i, fresh);
+        }
+        cp_async_commit();
+    };
+
+#pragma unroll
+    for (int s = 0; s < S; ++s) {
+        ek[s] = NONE;
+        if ((uint32_t)s < nch) fetch(s, ew[s], ek[s]);
+    }
+#pragma unroll
+    for (int s = 0; s < S - 1; ++s) {
+        request(s, ew[s], ek[s]);
+        ek[s] = NONE;
+        if ((uint32_t)(s + S) < nch) fetch(s + S, ew[s], ek[s]);
+    }
+    for (uint32_t c0 = 0; c0 < nch; c0 += S) {
+#pragma unroll
+        for (int s = 0; s < S; ++s) {
+            const uint32_t cc = c0 + s;
+            if (cc >= nch) break;
+            const int js = (s + S - 1) % S;  // slot of chunk cc + S - 1
+            request(js, ew[js], ek[js]);
+            ek[js] = NONE;
+            if (cc + 2 * S - 1 < nch) fetch(cc + 2 * S - 1, ew[js], ek[js]);
+            cp_async_wait<S - 1>();  // chunk cc's row has landed (this lane's own copies)
+            const uint32_t kk = sk[s];
+            const uint32_t mk = __shfl_sync(FULL, mask, kk & 31u);
+            if (kk == NONE) continue;
+            ++n_read;
+            const uint32_t d = sd[s], w = sw[s];
+            const uint32_t* rv = vs + (s * 32 + lane) * RW;  // v's row (swizzled copies)
+            const uint32_t* ru = xs + kk * RW;               // u's row
+            uint32_t* pv = P.V + (size_t)d * RW;
+            uint32_t changed = 0;
+#pragma unroll
+            for (int gi = 0; gi < RW / L::G; ++gi) {
+                const uint32_t act = group_mask<L>(mk, gi);
+                if (!act) continue;
+                uint32_t uu[L::G], cc2[L::G];
+#pragma unroll
+                for (int j = 0; j < L::G; ++j) {
+                    const uint32_t i = (uint32_t)(gi * L::G + j);
+                    uu[j] = ru[i];
+                    cc2[j] = rv[((i / RC::CW4) ^ swz) * RC::CW4 + i % RC::CW4];
+                }
+                changed |= L::relax(pv + gi * L::G, uu, cc2, w, act, n_edges, n_upd, P.err) << (gi * L::G * L::QPW);
+            }
+            if (changed) {
+                red_or(P.M + d, changed);                                 // v active for those queries
+                if (set_bits) red_or(P.bitmap + (d >> 5), 1u << (d & 31));  // union frontier bit
+            }
+        }
+    }
+    cp_async_wait<0>();
+}
+
+// The window's 32 rows (all Q queries) into shared memory, coalesced (RW words per row)
+template <class L>
+__device__ __forceinline__ void load_rows(const BParams& P, uint32_t* xs, uint32_t v, uint32_t i, uint32_t count) {
+    const uint32_t lane = threadIdx.x & 31;
+    __syncwarp();
+#pragma unroll
+    for (int r = 0; r < L::RW; ++r) {
+        const uint32_t f = r * 32 + lane;  // flat index row*RW + word
+        const uint32_t vr = __shfl_sync(FULL, v, f / L::RW);
+        xs[f] = (i + f / L::RW < count) ? ld_cg(P.V + (size_t)vr * L::RW + f % L::RW) : 0u;
+    }
+    __syncwarp();
+}
+
+// first list entry of the warp's edge range: 32-ary search over the list's edge offsets
+__device__ __forceinline__ uint32_t first_entry(const BParams& P, uint32_t count, uint32_t e0) {
+    const uint32_t lane = threadIdx.x & 31;
     uint32_t lo = 0, hi = count;
     while (hi - lo > 32) {
         const uint32_t step = (hi - lo + 31) / 32;
@@ -338,12 +565,22 @@ __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, ui
         hi = min(hi, nlo + step);
         lo = nlo;
     }
-    {
-        const uint32_t p = lo + lane;
-        const bool le = p < hi && ld_cg(P.lo + p) <= e0;
-        lo += 31 - __clz(__ballot_sync(FULL, le));
-    }
-    uint32_t i = lo, e = e0;
+    const uint32_t p = lo + lane;
+    const bool le = p < hi && ld_cg(P.lo + p) <= e0;
+    return lo + 31 - __clz(__ballot_sync(FULL, le));
+}
+
+// S2 over the compacted list: the iteration's E list edges split evenly over all warps; a warp
+// slides 32-entry windows (a hub row is shared by as many warps and CTAs as needed).
+template <int KIND, bool PACKED, class L>
+__device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, uint32_t E, uint32_t* xs, uint32_t* vs,
+                        bool set_bits, bool fresh, uint32_t& n_edges, uint32_t& n_upd, uint32_t& n_read) {
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t gw = blockIdx.x * BW + (threadIdx.x >> 5);
+    const uint64_t NW = (uint64_t)gridDim.x * BW;
+    const uint32_t e0 = (uint32_t)((uint64_t)E * gw / NW), e1 = (uint32_t)((uint64_t)E * (gw + 1) / NW);
+    if (e0 >= e1) return;
+    uint32_t i = first_entry(P, count, e0), e = e0;
     for (;;) {
         const uint32_t idx = i + lane;
         uint32_t off = E, base = 0, v = 0, mask = 0;
@@ -353,65 +590,10 @@ __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, ui
             mask = ld_cg(P.lm + idx);
             base = __ldg(g.ptr + v) - off;
         }
-        // the window's 32 source rows (all B queries) into shared memory, coalesced
-        __syncwarp();
-#pragma unroll
-        for (int r = 0; r < B; ++r) {
-            const uint32_t f = r * 32 + lane;  // flat index row*B + q
-            const uint32_t vr = __shfl_sync(FULL, v, f / B);
-            xs[f] = (i + f / B < count) ? ld_cg(P.V + (size_t)vr * B + f % B) : 0u;
-        }
-        __syncwarp();
+        load_rows<L>(P, xs, v, i, count);
         const uint32_t wend = (i + 32 < count) ? ld_cg(P.lo + i + 32) : E;
         const uint32_t ehi = min(e1, wend);
-        for (; e < ehi; e += 32 * U) {
-            uint32_t k[U], mk[U];
-            bool ok[U];
-            EdgeWord<PACKED> wd[U];
-#pragma unroll
-            for (int u = 0; u < U; ++u) {
-                const uint32_t t = e + u * 32 + lane;
-                uint32_t kk = 0;
-#pragma unroll
-                for (uint32_t st = 16; st > 0; st >>= 1)
-                    if (__shfl_sync(FULL, off, kk + st) <= t) kk += st;
-                k[u] = kk;
-                mk[u] = __shfl_sync(FULL, mask, kk);
-                const uint32_t a = __shfl_sync(FULL, base, kk) + t;
-                ok[u] = t < ehi;
-                if (ok[u]) wd[u].load(g, a);
-            }
-            uint32_t d[U], w[U];
-            Row<B> cur[U];
-#pragma unroll
-            for (int u = 0; u < U; ++u)
-                if (ok[u]) {
-                    wd[u].decode(P.dbits, P.dmask, d[u], w[u]);
-                    cur[u].load(P.V + (size_t)d[u] * B, fresh);
-                }
-#pragma unroll
-            for (int u = 0; u < U; ++u) {
-                if (!ok[u]) continue;
-                Row<B> xu;
-                xu.load_smem(xs + k[u] * B);
-                uint32_t changed = 0;
-#pragma unroll
-                for (int q = 0; q < B; ++q) {
-                    if (!((mk[u] >> q) & 1u)) continue;
-                    ++n_edges;
-                    const uint32_t cand = O::ext(xu.x[q], w[u]);
-                    if (O::better(cand, cur[u].x[q])) {                       // Needed(e(u,v)), query q
-                        O::edge_fn(P.V + (size_t)d[u] * B + q, cand);         // EdgeFunction
-                        changed |= 1u << q;
-                        ++n_upd;
-                    }
-                }
-                if (changed) {
-                    red_or(P.M + d[u], changed);                              // v active for those queries
-                    if (set_bits) red_or(P.bitmap + (d[u] >> 5), 1u << (d[u] & 31));  // union frontier bit
-                }
-            }
-        }
+        window_edges<KIND, PACKED, L>(P, g, xs, vs, off, base, mask, e, ehi, set_bits, fresh, n_edges, n_upd, n_read);
         if (ehi >= e1) break;
         e = ehi;
         i += 32;
@@ -420,36 +602,20 @@ __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, ui
 
 // ------------------------------------------------------------------ NEXT-1 pull (Reduced(E))
 // The list holds vertices v with uncertified queries (mask) and their IN-edge offsets; a lane
-// takes an in-edge (u -> v, w) of the edge-balanced split and, for each uncertified query q
-// with Val(u) reached, applies the Table 6 Needed / EdgeFunction to Val(v): all pushes INTO
-// uncertified vertices in one sweep, none into certified ones (their in-edges are removed).
-template <int KIND, bool PACKED, int B>
+// takes an in-edge (u -> v, w) of the edge-balanced split and, for each uncertified query q,
+// applies the Table 6 Needed / EdgeFunction to Val(v): all pushes INTO uncertified vertices in
+// one sweep, none into certified ones (their in-edges are removed).
+template <int KIND, bool PACKED, class L>
 __device__ void relax_pull(const BParams& P, uint32_t count, uint32_t E, uint32_t* xs, uint32_t& n_edges,
-                           uint32_t& n_upd) {
-    using O = Op<KIND>;
-    constexpr int U = 2;
+                           uint32_t& n_upd, uint32_t& n_read) {
+    constexpr int U = 2, RW = L::RW;
     const GraphView& g = P.R;
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t gw = blockIdx.x * BW + (threadIdx.x >> 5);
     const uint64_t NW = (uint64_t)gridDim.x * BW;
     const uint32_t e0 = (uint32_t)((uint64_t)E * gw / NW), e1 = (uint32_t)((uint64_t)E * (gw + 1) / NW);
     if (e0 >= e1) return;
-    uint32_t lo = 0, hi = count;
-    while (hi - lo > 32) {
-        const uint32_t step = (hi - lo + 31) / 32;
-        const uint32_t p = lo + lane * step;
-        const bool le = p < hi && ld_cg(P.lo + p) <= e0;
-        const uint32_t k = 31 - __clz(__ballot_sync(FULL, le));
-        const uint32_t nlo = lo + k * step;
-        hi = min(hi, nlo + step);
-        lo = nlo;
-    }
-    {
-        const uint32_t p = lo + lane;
-        const bool le = p < hi && ld_cg(P.lo + p) <= e0;
-        lo += 31 - __clz(__ballot_sync(FULL, le));
-    }
-    uint32_t i = lo, e = e0;
+    uint32_t i = first_entry(P, count, e0), e = e0;
     for (;;) {
         const uint32_t idx = i + lane;
         uint32_t off = E, base = 0, v = 0, mask = 0;
@@ -459,14 +625,7 @@ __device__ void relax_pull(const BParams& P, uint32_t count, uint32_t E, uint32_
             mask = ld_cg(P.lm + idx);
             base = __ldg(g.ptr + v) - off;
         }
-        __syncwarp();
-#pragma unroll
-        for (int r = 0; r < B; ++r) {  // current rows of the pulling vertices (for the Needed test)
-            const uint32_t f = r * 32 + lane;
-            const uint32_t vr = __shfl_sync(FULL, v, f / B);
-            xs[f] = (i + f / B < count) ? ld_cg(P.V + (size_t)vr * B + f % B) : 0u;
-        }
-        __syncwarp();
+        load_rows<L>(P, xs, v, i, count);  // current rows of the pulling vertices (Needed test)
         const uint32_t wend = (i + 32 < count) ? ld_cg(P.lo + i + 32) : E;
         const uint32_t ehi = min(e1, wend);
         for (; e < ehi; e += 32 * U) {
@@ -484,32 +643,29 @@ __device__ void relax_pull(const BParams& P, uint32_t count, uint32_t E, uint32_
                 mk[u] = __shfl_sync(FULL, mask, kk);
                 vk[u] = __shfl_sync(FULL, v, kk);
                 const uint32_t a = __shfl_sync(FULL, base, kk) + t;
-                ok[u] = t < ehi;
+                ok[u] = t < ehi && mk[u] != 0u;
                 if (ok[u]) wd[u].load(g, a);
             }
-            uint32_t src[U], w[U];
-            Row<B> xu[U];
-#pragma unroll
-            for (int u = 0; u < U; ++u)
-                if (ok[u]) {
-                    wd[u].decode(P.dbits, P.dmask, src[u], w[u]);
-                    xu[u].load(P.V + (size_t)src[u] * B, false);
-                }
 #pragma unroll
             for (int u = 0; u < U; ++u) {
                 if (!ok[u]) continue;
+                uint32_t src, w;
+                wd[u].decode(P.dbits, P.dmask, src, w);
+                ++n_read;
+                const uint32_t* ru = P.V + (size_t)src * RW;  // u's row (L1: a stale value is never better)
+                uint32_t* pv = P.V + (size_t)vk[u] * RW;
                 uint32_t changed = 0;
 #pragma unroll
-                for (int q = 0; q < B; ++q) {
-                    if (!((mk[u] >> q) & 1u)) continue;
-                    ++n_edges;
-                    if (xu[u].x[q] == O::INIT) continue;  // u unreached for q: nothing to pull
-                    const uint32_t cand = O::ext(xu[u].x[q], w[u]);
-                    if (O::better(cand, xs[k[u] * B + q])) {              // Needed(e(u,v)), query q
-                        O::edge_fn(P.V + (size_t)vk[u] * B + q, cand);    // EdgeFunction
-                        changed |= 1u << q;
-                        ++n_upd;
+                for (int gi = 0; gi < RW / L::G; ++gi) {
+                    const uint32_t act = group_mask<L>(mk[u], gi);
+                    if (!act) continue;
+                    uint32_t uu[L::G], cc2[L::G];
+#pragma unroll
+                    for (int j = 0; j < L::G; ++j) {
+                        uu[j] = ld_l1(ru + gi * L::G + j);
+                        cc2[j] = xs[k[u] * RW + gi * L::G + j];
                     }
+                    changed |= L::relax(pv + gi * L::G, uu, cc2, w, act, n_edges, n_upd, P.err) << (gi * L::G * L::QPW);
                 }
                 if (changed) red_or(P.M + vk[u], changed);  // v pushes onward for those queries
             }
@@ -530,63 +686,80 @@ __device__ __forceinline__ void block_add_split(unsigned long long* stats, int q
             atomicAdd(stats + (size_t)(q0 + b) * NSTAT + k, t / nq + (b == 0 ? t % nq : 0));
 }
 
-// Add a per-thread count to query (tid % B)'s counter k (grid-stride loops over [n][B] keep the
-// thread's query fixed because the stride is a multiple of B).
-template <int B>
+// Add a per-thread count to query (tid % Q)'s counter k (the thread's query is fixed in loops
+// whose stride is a multiple of Q).
+template <int Q>
 __device__ __forceinline__ void per_query_add(unsigned long long* stats, int q0, int nq, int k, unsigned long long c) {
 #pragma unroll
-    for (int o = B; o < 32; o <<= 1) c += __shfl_xor_sync(FULL, c, o);
+    for (int o = Q; o < 32; o <<= 1) c += __shfl_xor_sync(FULL, c, o);
     const uint32_t lane = threadIdx.x & 31;
-    if (lane < (uint32_t)B && (int)lane < nq && c) atomicAdd(stats + (size_t)(q0 + lane) * NSTAT + k, c);
+    if (lane < (uint32_t)Q && (int)lane < nq && c) atomicAdd(stats + (size_t)(q0 + lane) * NSTAT + k, c);
 }
 
-// V[v][q] -> dst[(q0+q)*n + v] for q < nq, 32 vertices per warp through shared memory
-template <int B>
+// value of query q at v, caller encoding
+template <class L>
+__device__ __forceinline__ uint32_t value_of(const uint32_t* V, uint32_t v, uint32_t q) {
+    return L::decode(ld_cg(V + (size_t)v * L::RW + q / L::QPW), q % L::QPW);
+}
+
+// rows -> dst[(q0+q)*n + v] for q < nq, 32 vertices per warp through shared memory
+template <class L>
 __device__ void transpose_out(const BParams& P, uint32_t* dst, int q0, int nq, uint32_t* xs) {
+    constexpr int RW = L::RW;
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t gw = blockIdx.x * BW + (threadIdx.x >> 5);
     const uint32_t NW = gridDim.x * BW;
     for (uint32_t v0 = gw * 32; v0 < P.n; v0 += NW * 32) {
         __syncwarp();
 #pragma unroll
-        for (int r = 0; r < B; ++r) {
+        for (int r = 0; r < RW; ++r) {
             const uint32_t f = r * 32 + lane;
-            const uint32_t v = v0 + f / B;
-            xs[(f / B) * (B + 1) + f % B] = v < P.n ? ld_cg(P.V + (size_t)v * B + f % B) : 0u;
+            const uint32_t v = v0 + f / RW;
+            xs[(f / RW) * (RW + 1) + f % RW] = v < P.n ? ld_cg(P.V + (size_t)v * RW + f % RW) : 0u;
         }
         __syncwarp();
         const uint32_t v = v0 + lane;
         if (v < P.n)
-            for (int q = 0; q < nq; ++q) dst[(size_t)(q0 + q) * P.n + v] = xs[lane * (B + 1) + q];
+            for (int q = 0; q < nq; ++q)
+                dst[(size_t)(q0 + q) * P.n + v] = L::decode(xs[lane * (RW + 1) + q / L::QPW], q % L::QPW);
     }
 }
 
-template <int KIND, bool PACKED, int B>
+template <class L>
+constexpr uint32_t xs_words() { return (32 * (L::RW + 1) + 3) & ~3u; }  // per warp, 16 B aligned
+template <class L>
+constexpr uint32_t vs_words() { return S_PIPE * 32 * L::RW; }
+
+template <int KIND, bool PACKED, class L>
 __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
-    using O = Op<KIND>;
+    constexpr int Q = L::Q, RW = L::RW;
     __shared__ uint32_t sm_cnt[2 * BW + 2];
     __shared__ unsigned long long sm_red[BW];
-    extern __shared__ uint32_t dsm[];  // per warp: 32*(B+1) words; then B*2K source hub values
-    uint32_t* xs = dsm + (threadIdx.x >> 5) * 32 * (B + 1);
-    uint32_t* sh = dsm + BW * 32 * (B + 1);
+    // dynamic shared memory: per warp xs (window rows / transpose tile), then per warp the
+    // S_PIPE-stage value-row ring vs, then Q*2*64 source hub values sh (certificates)
+    extern __shared__ __align__(16) uint32_t dsm[];
+    uint32_t* xs = dsm + (threadIdx.x >> 5) * xs_words<L>();
+    uint32_t* vs = dsm + BW * xs_words<L>() + (threadIdx.x >> 5) * vs_words<L>();
+    uint32_t* sh = dsm + BW * (xs_words<L>() + vs_words<L>());
     unsigned long long epoch = 0;
     const uint64_t tid = blockIdx.x * (uint64_t)BT + threadIdx.x;
     const uint64_t nthreads = (uint64_t)gridDim.x * BT;
     uint32_t ring = 0;
 
-    for (int q0 = 0; q0 < P.n_src; q0 += B) {
-        const int nq = min(B, P.n_src - q0);
+    for (int q0 = 0; q0 < P.n_src; q0 += Q) {
+        const int nq = min(Q, P.n_src - q0);
         // Alg 3 l.4, l.6 for every query of the batch; masks cleared
-        for (uint64_t i = tid; i < (uint64_t)P.n * B; i += nthreads) P.V[i] = O::INIT;
+        for (uint64_t i = tid; i < (uint64_t)P.n * RW; i += nthreads) P.V[i] = L::init_word();
         for (uint64_t v = tid; v < P.n; v += nthreads) P.M[v] = 0u;
         grid_sync(P.ctrl, epoch);
         for (int b = 0; b < nq; ++b) {
             const uint32_t s = __ldg(P.srcs + q0 + b);
             if (s >= P.n) {
-                if (tid == 0) atomicOr(P.err, 2u);
+                if (tid == 0) atomicOr(P.err, ERR_SOURCE);
                 continue;
             }
-            if (tid == 0) P.V[(size_t)s * B + b] = O::SRC;
+            uint32_t* col = P.V + b / L::QPW;
+            if (tid == 0) L::seed(col + (size_t)s * RW, b % L::QPW, L::src_val());
             // l.5, l.10: out-neighbours of s in G
             const uint32_t r0 = __ldg(P.G.ptr + s), r1 = __ldg(P.G.ptr + s + 1);
             for (uint64_t e = r0 + tid; e < r1; e += nthreads) {
@@ -594,7 +767,7 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
                 wd.load(P.G, (uint32_t)e);
                 uint32_t d, w;
                 wd.decode(P.dbits, P.dmask, d, w);
-                P.V[(size_t)d * B + b] = O::ext(O::SRC, w);
+                L::seed(col + (size_t)d * RW, b % L::QPW, L::nb_val(w));
                 red_or(P.M + d, 1u << b);
                 red_or(P.bitmap + (d >> 5), 1u << (d & 31));
             }
@@ -610,13 +783,13 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
         grid_sync(P.ctrl, epoch);
 
         int phase = P.two_phase ? 1 : 2;
-        bool predicate = false;
-        bool bits = true;  // the current frontier is in the bitmap (seeds set bits), else in M
-        bool pull = false; // this iteration is the NEXT-1 pull over uncertified vertices
-        uint32_t iters = 0, n_edges = 0, n_upd = 0;  // (edge, query) pairs of the whole batch
-        unsigned long long n_scan = 0;                // union edges read (every thread keeps the sum)
+        bool predicate = false;  // this iteration's S1 seeds Active with the impacted vertices
+        bool bits = true;        // the current frontier is in the bitmap (seeds set bits), else in M
+        bool pull = false;       // this iteration is the NEXT-1 pull over uncertified vertices
+        uint32_t iters = 0, n_edges = 0, n_upd = 0, n_read = 0;  // (edge, query) pairs / edge reads
         for (;;) {
             const GraphView& g = (phase == 1) ? P.C : P.G;
+            const bool fresh = (P.fresh >> (phase - 1)) & 1u;
             const int slot = ring & 3;
             unsigned long long* ctr = P.ctrl + CT0 + CTS * slot;
             if (tid == 0) {
@@ -625,7 +798,7 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
             }
             const unsigned long long t_s0 = (P.trace && tid == 0) ? global_ns() : 0ull;
             const int mode = pull ? F_UNCERT : predicate ? F_IMPACTED : bits ? F_BITS : F_MASKS;
-            compact_b<KIND, B>(P, pull ? P.R : g, mode, sh, nq, ctr + CT_LIST, ctr + CT_ACTIVE, sm_cnt);
+            compact<KIND, L>(P, pull ? P.R : g, mode, sh, nq, ctr + CT_LIST, ctr + CT_ACTIVE, sm_cnt);
             grid_sync(P.ctrl, epoch);
             ++ring;
             const unsigned long long ce = ld_cg64(ctr + CT_LIST);
@@ -648,29 +821,29 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
                 pull = false;
                 bits = false;
             }
-            n_scan += E;
             if (E == 0) {
-                if (P.stats && tid == 0 && n_scan)
-                    for (int b = 0; b < nq; ++b)
-                        atomicAdd(P.stats + (size_t)(q0 + b) * NSTAT + (phase == 1 ? ST_S1 : ST_S2),
-                                  n_scan / nq + (b == 0 ? n_scan % nq : 0));
-                n_scan = 0;
                 if (P.stats) {  // batch totals, attributed evenly to the batch's queries
                     block_add_split(P.stats, q0, nq, phase == 1 ? ST_E1 : ST_E2, n_edges, sm_red);
                     block_add_split(P.stats, q0, nq, phase == 1 ? ST_U1 : ST_U2, n_upd, sm_red);
+                    block_add_split(P.stats, q0, nq, phase == 1 ? ST_S1 : ST_S2, n_read, sm_red);
                     if (tid < (uint64_t)nq)
                         atomicAdd(P.stats + (size_t)(q0 + tid) * NSTAT + (phase == 1 ? ST_IT1 : ST_IT2),
                                   (unsigned long long)iters);
                 }
-                n_edges = n_upd = 0;
+                n_edges = n_upd = n_read = 0;
                 iters = 0;
                 if (phase == 1) {
-                    if (P.p1) transpose_out<B>(P, P.p1, q0, nq, xs);
-                    if (P.stats) {  // impacted per query (Alg 3 l.15); stride is a multiple of B: q fixed
+                    if (P.p1) transpose_out<L>(P, P.p1, q0, nq, xs);
+                    if (P.stats) {  // impacted per query (Alg 3 l.15); the thread's query q is fixed
+                        const uint32_t q = (uint32_t)(tid % Q);
+                        const uint32_t init = L::decode(L::init_word(), 0);
                         unsigned long long c = 0;
-                        for (uint64_t i = tid; i < (uint64_t)P.n * B; i += nthreads) c += ld_cg(P.V + i) != O::INIT;
-                        per_query_add<B>(P.stats, q0, nq, ST_IMP, c);
+                        for (uint64_t v = tid / Q; v < P.n; v += nthreads / Q)
+                            c += value_of<L>(P.V, (uint32_t)v, q) != init;
+                        per_query_add<Q>(P.stats, q0, nq, ST_IMP, c);
                     }
+                    // the p1 / impacted reads must finish before phase 2 updates V
+                    if (P.p1 || P.stats) grid_sync(P.ctrl, epoch);
                     phase = 2;
                     if (P.reduced) pull = true;   // Reduced(E): pull into uncertified vertices
                     else predicate = true;        // Active <- impacted vertices (l.15)
@@ -679,89 +852,108 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
                 break;
             }
             if (pull) {  // NEXT-1: one pull sweep, then push from the vertices it changed (masks in M)
-                relax_pull<KIND, PACKED, B>(P, count, E, xs, n_edges, n_upd);
+                relax_pull<KIND, PACKED, L>(P, count, E, xs, n_edges, n_upd, n_read);
                 pull = false;
                 bits = false;
-                grid_sync(P.ctrl, epoch);
-                if (P.trace && tid == 0 && tr < P.trace_cap) P.trace[5ull * tr + 2] = global_ns();
-                ++iters;
-                continue;
+            } else {
+                // small frontier: its S2 sets frontier bits (few reds) and the next S1 reads the
+                // bitmap; large frontier: no bitmap reds (they contend in L2), the next S1 scans M
+                bits = count < P.bits_below;
+                relax_b<KIND, PACKED, L>(P, g, count, E, xs, vs, bits, fresh, n_edges, n_upd, n_read);
+                predicate = false;
             }
-            // small frontier: its S2 sets frontier bits (few reds) and the next S1 reads the bitmap;
-            // large frontier: no bitmap reds (they contend in L2), the next S1 scans M instead
-            bits = count < P.bits_below;
-            relax_b<KIND, PACKED, B>(P, g, count, E, xs, bits, (P.fresh >> (phase - 1)) & 1u, n_edges, n_upd);
-            predicate = false;
             grid_sync(P.ctrl, epoch);
             if (P.trace && tid == 0 && tr < P.trace_cap) P.trace[5ull * tr + 2] = global_ns();
             if (++iters > P.max_iters) {
-                if (tid == 0) atomicOr(P.err, 1u);
+                if (tid == 0) atomicOr(P.err, ERR_ITERS);
                 return;
             }
         }
-        transpose_out<B>(P, P.out, q0, nq, xs);
-        if (P.stats) {  // reached / precise per query (thread's query b = tid % B is fixed)
-            const uint32_t b = (uint32_t)(tid % B);
-            const uint32_t sb = (int)b < nq ? __ldg(P.srcs + q0 + b) : 0xffffffffu;
+        transpose_out<L>(P, P.out, q0, nq, xs);
+        if (P.stats) {  // reached / precise per query (the thread's query q is fixed)
+            const uint32_t q = (uint32_t)(tid % Q);
+            const uint32_t sb = (int)q < nq ? __ldg(P.srcs + q0 + q) : 0xffffffffu;
+            const uint32_t init = L::decode(L::init_word(), 0);
             unsigned long long r = 0, pr = 0;
-            for (uint64_t i = tid; i < (uint64_t)P.n * B; i += nthreads) {
-                const uint32_t v = (uint32_t)(i / B);
-                const uint32_t fv = ld_cg(P.V + i);
-                if ((int)b < nq && v != sb && fv != O::INIT) {
-                    ++r;
-                    if (P.p1 && ld_cg(P.p1 + (size_t)(q0 + b) * P.n + v) == fv) ++pr;
+            if ((int)q < nq)
+                for (uint64_t v = tid / Q; v < P.n; v += nthreads / Q) {
+                    const uint32_t fv = value_of<L>(P.V, (uint32_t)v, q);
+                    if (v != sb && fv != init) {
+                        ++r;
+                        if (P.p1 && ld_cg(P.p1 + (size_t)(q0 + q) * P.n + v) == fv) ++pr;
+                    }
                 }
-            }
-            per_query_add<B>(P.stats, q0, nq, ST_REACH, r);
-            per_query_add<B>(P.stats, q0, nq, ST_PREC, pr);
+            per_query_add<Q>(P.stats, q0, nq, ST_REACH, r);
+            per_query_add<Q>(P.stats, q0, nq, ST_PREC, pr);
         }
         grid_sync(P.ctrl, epoch);  // V / M / bitmap are reused by the next batch
     }
 }
 
-template <int KIND, bool PACKED, int B>
+template <int KIND, bool PACKED, int LW>
 void launch_b(const BParams& P, int sms, cudaStream_t s) {
-    const size_t smem = ((size_t)BW * 32 * (B + 1) + (size_t)B * 2 * 64) * sizeof(uint32_t);
+    using L = typename LanesOf<LW, KIND>::T;
+    const size_t smem = ((size_t)BW * (xs_words<L>() + vs_words<L>()) + (size_t)L::Q * 2 * 64) * sizeof(uint32_t);
     static int bps = 0;
     if (!bps) {
         if (smem > 48 * 1024)
-            CGB_CUDA(cudaFuncSetAttribute(batch_kernel<KIND, PACKED, B>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+            CGB_CUDA(cudaFuncSetAttribute(batch_kernel<KIND, PACKED, L>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                           (int)smem));
-        CGB_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, batch_kernel<KIND, PACKED, B>, BT, smem));
+        CGB_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, batch_kernel<KIND, PACKED, L>, BT, smem));
         CGB_CHECK(bps > 0, CG_EUNSUPPORTED, "batch kernel cannot be resident");
     }
     void* args[] = {(void*)&P};
-    CGB_CUDA(cudaLaunchCooperativeKernel((const void*)batch_kernel<KIND, PACKED, B>, dim3(bps * sms), dim3(BT), args,
+    CGB_CUDA(cudaLaunchCooperativeKernel((const void*)batch_kernel<KIND, PACKED, L>, dim3(bps * sms), dim3(BT), args,
                                          smem, s));
     count_launch();
 }
 
-template <bool PACKED, int B>
-void launch_kind_b(int kind, const BParams& P, int sms, cudaStream_t s) {
+template <bool PACKED>
+void launch_kind_b(int kind, int lw, const BParams& P, int sms, cudaStream_t s) {
     switch (kind) {
-    case CG_SSSP: launch_b<CG_SSSP, PACKED, B>(P, sms, s); break;
-    case CG_SSWP: launch_b<CG_SSWP, PACKED, B>(P, sms, s); break;
-    case CG_SSNP: launch_b<CG_SSNP, PACKED, B>(P, sms, s); break;
-    case CG_VITERBI: launch_b<CG_VITERBI, PACKED, B>(P, sms, s); break;
-    case CG_BFS: launch_b<CG_BFS, PACKED, B>(P, sms, s); break;
-    case CG_REACH: launch_b<CG_REACH, PACKED, B>(P, sms, s); break;
+    case CG_SSSP:
+        if (lw == 16) launch_b<CG_SSSP, PACKED, 16>(P, sms, s);
+        else launch_b<CG_SSSP, PACKED, 32>(P, sms, s);
+        break;
+    case CG_SSWP:
+        if (lw == 16) launch_b<CG_SSWP, PACKED, 16>(P, sms, s);
+        else launch_b<CG_SSWP, PACKED, 32>(P, sms, s);
+        break;
+    case CG_SSNP:
+        if (lw == 16) launch_b<CG_SSNP, PACKED, 16>(P, sms, s);
+        else launch_b<CG_SSNP, PACKED, 32>(P, sms, s);
+        break;
+    case CG_VITERBI: launch_b<CG_VITERBI, PACKED, 32>(P, sms, s); break;
+    case CG_BFS:
+        if (lw == 16) launch_b<CG_BFS, PACKED, 16>(P, sms, s);
+        else launch_b<CG_BFS, PACKED, 32>(P, sms, s);
+        break;
+    case CG_REACH:
+        if (lw == 1) launch_b<CG_REACH, PACKED, 1>(P, sms, s);
+        else launch_b<CG_REACH, PACKED, 32>(P, sms, s);
+        break;
     default: throw Error(CG_EINVAL, "bad kind");
     }
 }
 
-}  // namespace
-
-int batch_width() {
-    const char* e = getenv("CG_BATCH");
-    const int b = e ? atoi(e) : 16;
-    return (b == 8 || b == 16 || b == 32) ? b : 0;  // 0 (or anything else): single-query engine
+// Value lanes of a call: f16 for SSSP / SSWP / SSNP / BFS (SSWP / SSNP need w_max <= 2048, SSSP
+// w_max <= 2048; SSSP / BFS fall back to u32 lanes on a lane overflow), one bit for REACH, u32
+// for Viterbi (CG_LANES=32 forces u32 lanes for every kind).
+int lane_width(const Graph& G, int kind) {
+    const char* e = getenv("CG_LANES");
+    if (e && atoi(e) == 32) return 32;
+    if (kind == CG_REACH) return 1;
+    if (kind == CG_BFS) return 16;
+    if ((kind == CG_SSSP || kind == CG_SSWP || kind == CG_SSNP) && G.w_max <= 2048) return 16;
+    return 32;
 }
 
-void run_queries_batched(Graph& G, const QueryCall& c, int B, cudaStream_t s, std::vector<cg_stats>* stats) {
+void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::vector<cg_stats>* stats,
+                    uint32_t* err_out) {
     BatchSpace& w = G.bs;
     const uint32_t words = (G.n + 31) / 32;
-    if (w.n != G.n || w.B != (uint32_t)B) {
-        w.V.alloc((size_t)G.n * B, s);
+    if (w.n != G.n) {
+        w.V.alloc((size_t)G.n * 16, s);  // the widest row: 16 u32 words
         w.M.alloc(G.n ? G.n : 1, s);
         w.bitmap.alloc(words ? words : 1, s);
         w.lv.alloc(G.n ? G.n : 1, s);
@@ -770,8 +962,9 @@ void run_queries_batched(Graph& G, const QueryCall& c, int B, cudaStream_t s, st
         w.ctrl.alloc(CT0 + CTS * 4, s);
         w.err.alloc(1, s);
         w.n = G.n;
-        w.B = (uint32_t)B;
+        w.B = 16;
     }
+    const int Q = lw == 32 ? 16 : 32;
     DevBuf<unsigned long long> st;
     if (stats) st.alloc((size_t)c.n_src * NSTAT, s);
     BParams P{};
@@ -784,12 +977,14 @@ void run_queries_batched(Graph& G, const QueryCall& c, int B, cudaStream_t s, st
     P.R = view(G.gr);
     {   // NEXT-1 (Reduced(E) pull) after phase 1 for the kinds with a certificate; CG_REDUCED is a
         // bitmask over cg_kind.  Default REACH only: its certificate (reached = final) leaves only
-        // unreachable vertices; the SSWP / SSNP / SSSP certificates are exact but, united over a
-        // 16-query batch, leave ~99 % of the vertices uncertified for some query (measured, C2).
+        // unreachable vertices; the SSWP / SSNP / SSSP certificates (u32 lanes) are exact but,
+        // united over a 16-query batch, leave ~99 % of the vertices uncertified for some query
+        // (measured, C2).
         const char* e = getenv("CG_REDUCED");
         const unsigned mask = e ? (unsigned)strtoul(e, nullptr, 0) : (1u << CG_REACH);
         const Core& core = G.core[core_slot(c.kind)];
-        const bool has_cert = c.kind == CG_REACH || (core.hub_k > 0 && core.hub_k <= 64 && core.hub_vals.get());
+        const bool hub_cert = lw == 32 && core.hub_k > 0 && core.hub_k <= 64 && core.hub_vals.get();
+        const bool has_cert = c.kind == CG_REACH || hub_cert;
         P.reduced = c.two_phase && c.core_adj == &core.adj && ((mask >> c.kind) & 1u) && has_cert;
         if (P.reduced && c.kind != CG_REACH) {
             P.HB = core.hub_vals.get();
@@ -830,15 +1025,9 @@ void run_queries_batched(Graph& G, const QueryCall& c, int B, cudaStream_t s, st
         CGB_CUDA(cudaMemsetAsync(trace.get(), 0, trace.bytes(), s));
         P.trace = trace.get();
     }
-    if (G.packed) {
-        if (B == 8) launch_kind_b<true, 8>(c.kind, P, G.num_sms, s);
-        else if (B == 16) launch_kind_b<true, 16>(c.kind, P, G.num_sms, s);
-        else launch_kind_b<true, 32>(c.kind, P, G.num_sms, s);
-    } else {
-        if (B == 8) launch_kind_b<false, 8>(c.kind, P, G.num_sms, s);
-        else if (B == 16) launch_kind_b<false, 16>(c.kind, P, G.num_sms, s);
-        else launch_kind_b<false, 32>(c.kind, P, G.num_sms, s);
-    }
+    if (G.packed) launch_kind_b<true>(c.kind, lw, P, G.num_sms, s);
+    else launch_kind_b<false>(c.kind, lw, P, G.num_sms, s);
+    CGB_CUDA(cudaMemcpyAsync(err_out, w.err.get(), 4, cudaMemcpyDeviceToHost, s));
     if (tracing) {
         std::vector<unsigned long long> h(5ull * P.trace_cap);
         CGB_CUDA(cudaMemcpyAsync(h.data(), trace.get(), trace.bytes(), cudaMemcpyDeviceToHost, s));
@@ -847,20 +1036,16 @@ void run_queries_batched(Graph& G, const QueryCall& c, int B, cudaStream_t s, st
         for (uint32_t i = 0; i < P.trace_cap && h[5 * i]; ++i) {
             const unsigned long long* t = h.data() + 5 * i;
             if (!t0) t0 = t[0];
-            fprintf(stderr, "CG_TRACE kind=%d B=%d it=%u q0=%llu phase=%llu list=%llu active=%llu edges=%llu "
-                    "t=%.1f s1=%.1f s2=%.1f us\n", c.kind, B, i, (t[3] >> 32) & 0x3fffffffull, t[3] >> 62,
+            fprintf(stderr, "CG_TRACE kind=%d Q=%d lanes=%d it=%u q0=%llu phase=%llu list=%llu active=%llu edges=%llu "
+                    "t=%.1f s1=%.1f s2=%.1f us\n", c.kind, Q, lw, i, (t[3] >> 32) & 0x3fffffffull, t[3] >> 62,
                     t[3] & 0xffffffffull, t[4] >> 32, t[4] & 0xffffffffull, (t[0] - t0) / 1e3, (t[1] - t[0]) / 1e3,
                     t[2] ? (t[2] - t[1]) / 1e3 : 0.0);
         }
     }
     if (stats) {
         std::vector<unsigned long long> h((size_t)c.n_src * NSTAT);
-        uint32_t err = 0;
         CGB_CUDA(cudaMemcpyAsync(h.data(), st.get(), st.bytes(), cudaMemcpyDeviceToHost, s));
-        CGB_CUDA(cudaMemcpyAsync(&err, w.err.get(), 4, cudaMemcpyDeviceToHost, s));
         CGB_CUDA(cudaStreamSynchronize(s));
-        CGB_CHECK(!(err & 2u), CG_EINVAL, "source id >= n");
-        CGB_CHECK(!(err & 1u), CG_EINTERNAL, "iteration bound exceeded");
         stats->resize(c.n_src);
         for (int qq = 0; qq < c.n_src; ++qq) {
             const unsigned long long* x = h.data() + (size_t)qq * NSTAT;
@@ -878,7 +1063,36 @@ void run_queries_batched(Graph& G, const QueryCall& c, int B, cudaStream_t s, st
             o.precise_p1 = P.p1 ? (int64_t)x[ST_PREC] : -1;
             o.scanned_p1 = (int64_t)x[ST_S1];
             o.scanned_p2 = (int64_t)x[ST_S2];
+            o.batch_queries = Q;
+            o.row_bytes = lw == 1 ? 4 : 64;
         }
+    }
+}
+
+}  // namespace
+
+int batch_width() {
+    const char* e = getenv("CG_BATCH");
+    return (e && atoi(e) == 0) ? 0 : 16;  // CG_BATCH=0: single-query engine (engine.cu)
+}
+
+void run_queries_batched(Graph& G, const QueryCall& c, int, cudaStream_t s, std::vector<cg_stats>* stats) {
+    const int lw = lane_width(G, c.kind);
+    uint32_t* err = G.bs.err_host();
+    run_batched_lw(G, c, lw, s, stats, err);
+    // f16 SSSP / BFS lanes must know about a lane overflow before the results are trusted: such
+    // a call synchronises once and re-runs with u32 lanes if any candidate reached 2048
+    if (lw == 16 && (c.kind == CG_BFS || c.kind == CG_SSSP)) {
+        CGB_CUDA(cudaStreamSynchronize(s));
+        if (*err & ERR_LANE_OVERFLOW) {
+            *err = 0;
+            run_batched_lw(G, c, 32, s, stats, err);
+        }
+    }
+    if (stats) {
+        CGB_CUDA(cudaStreamSynchronize(s));
+        CGB_CHECK(!(*err & ERR_SOURCE), CG_EINVAL, "source id >= n");
+        CGB_CHECK(!(*err & ERR_ITERS), CG_EINTERNAL, "iteration bound exceeded");
     }
 }
 

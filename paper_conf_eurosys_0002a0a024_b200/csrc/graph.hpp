@@ -56,14 +56,26 @@ struct Workspace {
     uint32_t stats_cap = 0;
 };
 
-struct BatchSpace {         // engine_batch.cu workspace (B queries per pass)
+struct BatchSpace {         // engine_batch.cu workspace (one batch of queries per pass)
     uint32_t n = 0, B = 0;
-    DevBuf<uint32_t> V;         // [n][B] values
+    DevBuf<uint32_t> V;         // [n][row words] value rows
     DevBuf<uint32_t> M;         // [n] active-query masks
     DevBuf<uint32_t> bitmap;    // union frontier
     DevBuf<uint32_t> lv, lo, lm;
     DevBuf<unsigned long long> ctrl;
     DevBuf<uint32_t> err;
+    uint32_t* err_h = nullptr;  // pinned host copy of err
+    uint32_t* err_host() {
+        if (!err_h) CGB_CUDA(cudaMallocHost(&err_h, sizeof(uint32_t)));
+        *err_h = 0;
+        return err_h;
+    }
+    BatchSpace() = default;
+    BatchSpace(const BatchSpace&) = delete;
+    BatchSpace& operator=(const BatchSpace&) = delete;
+    ~BatchSpace() {
+        if (err_h) cudaFreeHost(err_h);
+    }
 };
 
 struct Graph {

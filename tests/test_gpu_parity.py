@@ -111,6 +111,39 @@ def test_long_chain_loop_control():
                    modes=("full",))
 
 
+def test_f16_lane_overflow_falls_back():
+    """SSSP and BFS run in binary16 lanes, exact for integers below 2048; a candidate of 2048 or
+    more sets the lane-overflow flag and the call re-runs in u32 lanes: a 2500-vertex chain
+    (levels / distances up to 2499) plus shortcuts, 2Phase and FULL, several sources."""
+    n = 2500
+    src = np.concatenate([np.arange(n - 1), [0, 1, 2]]).astype(np.uint32)
+    dst = np.concatenate([np.arange(1, n), [1300, 1450, 2499]]).astype(np.uint32)
+    w = np.ones(src.size, np.uint32)
+    _check_queries(n, src, dst, w, np.array([0, 5, 100, 400, 2490], np.uint32), kinds=("sssp", "bfs", "reach", "sswp"),
+                   K=4)
+
+
+def test_wide_weights_use_u32_lanes():
+    """SSWP / SSNP values are edge weights: binary16 lanes (32 queries per pass) only while
+    w_max <= 2048; wider weights run in u32 lanes (16 per pass, cg_stats.batch_queries tells
+    which), with the same results."""
+    rng = np.random.default_rng(12)
+    n, m = 3000, 24000
+    src, dst = rng.integers(0, n, m).astype(np.uint32), rng.integers(0, n, m).astype(np.uint32)
+    for w_hi, qb in ((2000, 32), (5000, 16)):
+        w = rng.integers(1, w_hi + 1, m).astype(np.uint32)
+        g, og = both(n, src, dst, w)
+        sources = np.arange(0, 40, dtype=np.uint32)
+        for kind in ("sswp", "ssnp"):
+            g.build(kind, K=8)
+            out, st = g.query(kind, to_dev(sources), mode="2phase", stats=True)
+            out = to_np(out)
+            assert all(x["batch_queries"] == qb for x in st), (kind, w_hi)
+            for i, s in enumerate(sources):
+                assert_values_equal(out[i], oracle.query(kind, og, int(s)), kind, f"w<={w_hi} {kind} s={s}")
+        g.close()
+
+
 def test_star_hub_chunks():
     """A hub with 10^6 out-edges exercises the multi-CTA chunk tier (rows >= kBigThreshold)."""
     leaves = 1_000_000
@@ -240,18 +273,24 @@ def test_dense_and_sparse_iterations(dense_div, monkeypatch):
                 assert_values_equal(out[i], oracle.query(kind, og, int(s)), kind, f"{kind}/{mode}/div={dense_div}/s={s}")
 
 
-@pytest.mark.parametrize("batch", ["0", "8", "16", "32"])
-def test_single_and_batched_engines(batch, monkeypatch):
-    """CG_BATCH=0 runs every source through the single-query engine; 8/16/32 run B sources per
-    pass (NEXT-2, values laid out [n][B]).  A ragged tail (13 sources), all kinds, both modes,
+@pytest.mark.parametrize("engine", ["single", "u32", "packed"])
+def test_single_and_batched_engines(engine, monkeypatch):
+    """CG_BATCH=0 runs every source through the single-query engine; otherwise sources run in
+    batches (NEXT-2): "u32" forces u32 value lanes (16 queries per pass, CG_LANES=32), "packed"
+    is the default (binary16 lanes for SSSP / SSWP / SSNP / BFS, bit lanes for REACH, 32 per pass).  Ragged
+    tails (45 sources: 2 full u32 passes + 13; 1 packed pass + 13), all kinds, both modes,
     phase-1 values and the unique per-query counts must match the oracle."""
-    monkeypatch.setenv("CG_BATCH", batch)
+    if engine == "single":
+        monkeypatch.setenv("CG_BATCH", "0")
+    elif engine == "u32":
+        monkeypatch.setenv("CG_LANES", "32")
+    batch = engine
     n, m = 1 << 14, 16 << 14
     src, dst, w = gen.rmat(n, m, w_max=27, seed=21)
     g, og = both(n, src, dst, w)
     ogr = oracle.transpose(og)
     hubs = oracle.hubs_topdeg(og, ogr, 20)
-    sources = np.concatenate([[0, 0], gen.sample_sources(n, src, dst, 11, seed=4)]).astype(np.uint32)
+    sources = np.concatenate([[0, 0], gen.sample_sources(n, src, dst, 43, seed=4)]).astype(np.uint32)
     for kind in KINDS:
         g.build(kind, K=20)
         cg = oracle.subgraph(og, oracle.cg_for_kind(kind, og, ogr, hubs))
@@ -271,7 +310,6 @@ def test_single_and_batched_engines(batch, monkeypatch):
 def test_batched_frontier_modes(bits_below, monkeypatch):
     """The batched engine keeps the union frontier either as bitmap bits set by S2 or as the
     per-vertex query masks scanned by S1 (chosen per iteration); force each everywhere."""
-    monkeypatch.setenv("CG_BATCH", "16")
     monkeypatch.setenv("CG_BITS_BELOW", bits_below)
     n, m = 1 << 15, 16 << 15
     src, dst, w = gen.rmat(n, m, w_max=15, seed=33)
@@ -285,12 +323,15 @@ def test_batched_frontier_modes(bits_below, monkeypatch):
                 assert_values_equal(out[i], oracle.query(kind, og, int(s)), kind, f"bits<{bits_below} {kind} {mode}")
 
 
-@pytest.mark.parametrize("reduced", ["0", "0x3f"])
-def test_reduced_pull_completion(reduced, monkeypatch):
+@pytest.mark.parametrize("reduced,lanes", [("0", ""), ("0x3f", ""), ("0x3f", "32")])
+def test_reduced_pull_completion(reduced, lanes, monkeypatch):
     """NEXT-1: phase 2 = one pull sweep over the in-edges of vertices whose phase-1 value is not
     certified (Theorem 1 P:1321-1371 and its bottleneck analogs; REACH: the lattice top), then
-    push.  Off (0) and on for every kind that has a certificate (0x3f): identical to the oracle."""
+    push.  Off (0) and on for every kind that has a certificate (0x3f; the hub certificates need
+    u32 lanes, forced by CG_LANES=32): identical to the oracle."""
     monkeypatch.setenv("CG_REDUCED", reduced)
+    if lanes:
+        monkeypatch.setenv("CG_LANES", lanes)
     n, m = 1 << 15, 16 << 15
     src, dst, w = gen.rmat(n, m, w_max=9, seed=44)
     g, og = both(n, src, dst, w)
