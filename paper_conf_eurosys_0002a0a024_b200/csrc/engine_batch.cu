@@ -78,10 +78,10 @@ struct BParams {
 //   src_val(), nb_val(w) SourceInitVal and SourceInitVal (+) w, encoded (Alg 3 l.5, l.8)
 //   relax(p, uw, cw, w, act, ...)  Process + EdgeFunction of one word (Alg 3 l.22-27): the lanes
 //       of act whose candidate ext(uw, w) is better than cw; returns the changed lanes
-template <int KIND>
-struct Lanes32 {  // one u32 per query (Table 6 types)
+template <int KIND, int QN>
+struct Lanes32 {  // one u32 per query (Table 6 types), QN queries per pass
     using O = Op<KIND>;
-    static constexpr int Q = 16, QPW = 1, RW = 16, G = 1;
+    static constexpr int Q = QN, QPW = 1, RW = QN, G = 1;
     __device__ static uint32_t init_word() { return O::INIT; }
     __device__ static uint32_t decode(uint32_t x, uint32_t) { return x; }
     __device__ static uint32_t live(uint32_t x) { return x != O::INIT; }
@@ -192,7 +192,8 @@ struct LanesBit {
 };
 
 template <int LW, int KIND> struct LanesOf;
-template <int KIND> struct LanesOf<32, KIND> { using T = Lanes32<KIND>; };
+template <int KIND> struct LanesOf<32, KIND> { using T = Lanes32<KIND, 16>; };  // u32 fallback: 16 per pass
+template <int KIND> struct LanesOf<33, KIND> { using T = Lanes32<KIND, 32>; };  // Viterbi: 32 per pass (128 B rows)
 template <int KIND> struct LanesOf<16, KIND> { using T = Lanes16<KIND>; };
 template <int KIND> struct LanesOf<1, KIND> { using T = LanesBit; };
 
@@ -202,13 +203,25 @@ __device__ __forceinline__ uint32_t group_mask(uint32_t mask, int i) {  // the l
     return LG >= 32 ? mask : (mask >> (i * LG)) & ((1u << LG) - 1u);
 }
 
-// queries with a non-InitVal value at v (L2 reads: values other SMs update)
+// queries with a non-InitVal value at v (L2 reads: values other SMs update; 16 B vector loads)
 template <class L>
 __device__ __forceinline__ uint32_t row_live(const uint32_t* V, uint32_t v) {
     const uint32_t* r = V + (size_t)v * L::RW;
     uint32_t m = 0;
+    if constexpr (L::RW % 4 == 0) {
 #pragma unroll
-    for (int i = 0; i < L::RW; ++i) m |= L::live(ld_cg(r + i)) << (i * L::QPW);
+        for (int i = 0; i < L::RW / 4; ++i) {
+            uint4 x;
+            asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];"
+                         : "=r"(x.x), "=r"(x.y), "=r"(x.z), "=r"(x.w)
+                         : "l"(reinterpret_cast<const uint4*>(r) + i));
+            m |= (L::live(x.x) | L::live(x.y) << L::QPW | L::live(x.z) << (2 * L::QPW) | L::live(x.w) << (3 * L::QPW))
+                 << (4 * i * L::QPW);
+        }
+    } else {
+#pragma unroll
+        for (int i = 0; i < L::RW; ++i) m |= L::live(ld_cg(r + i)) << (i * L::QPW);
+    }
     return m;
 }
 
@@ -273,17 +286,16 @@ __device__ uint32_t uncertified(const BParams& P, const uint32_t* sh, int nq, ui
 }
 
 // ------------------------------------------------------------------ S1 (union frontier)
-// mode: F_BITS (frontier bits set by S2), F_MASKS (frontier = {v : M[v] != 0}), F_IMPACTED
-// (Alg 3 l.15: v active for q iff Val(v) != InitVal), F_UNCERT (NEXT-1: v active for its
-// uncertified queries; degrees are then in-degrees, g = G^R).
-// Pass 1 counts the active vertices with edges and their edges per warp and reserves the CTA's
-// list range with ONE 64-bit atomicAdd; pass 2 writes (v, edge offset, query mask) in vertex
-// order, consuming the masks and the bitmap bits.
+// S1 modes: F_BITS (small frontiers: bitmap bits set by S2), F_MASKS (frontier = {v : M[v] != 0}),
+// F_IMPACTED (Alg 3 l.15: v active for q iff Val(v) != InitVal), F_UNCERT (NEXT-1: v active for
+// its uncertified queries; degrees are then in-degrees, g = G^R).  compact_bits (F_BITS): pass 1
+// counts the active vertices with edges and their edges per warp and reserves the CTA's list
+// range with ONE 64-bit atomicAdd; pass 2 writes (v, edge offset, query mask) in vertex order,
+// consuming the masks and the bitmap bits.
 enum { F_BITS = 0, F_MASKS = 1, F_IMPACTED = 2, F_UNCERT = 3 };
 
-template <int KIND, class L>
-__device__ void compact(const BParams& P, const GraphView& g, int mode, const uint32_t* sh, int nq,
-                        unsigned long long* cnt_slot, unsigned long long* act_slot, uint32_t* sm) {
+__device__ void compact_bits(const BParams& P, const GraphView& g, unsigned long long* cnt_slot,
+                             unsigned long long* act_slot, uint32_t* sm) {
     const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const uint64_t W = P.words;
     const uint32_t w0 = (uint32_t)(W * blockIdx.x / gridDim.x), w1 = (uint32_t)(W * (blockIdx.x + 1) / gridDim.x);
@@ -293,39 +305,7 @@ __device__ void compact(const BParams& P, const GraphView& g, int mode, const ui
     for (uint32_t g0 = w0 + warp * 32; g0 < w1; g0 += BW * 32) {
         const uint32_t wi = g0 + lane;
         uint32_t word = 0;
-        if (mode == F_IMPACTED) {  // Alg 3 l.15 for every query of the batch
-            for (uint32_t j = 0; j < 32; ++j) {
-                const uint32_t v = (g0 + j) * 32 + lane;
-                const bool act = g0 + j < w1 && v < P.n && row_live<L>(P.V, v) != 0;
-                const uint32_t bits = __ballot_sync(FULL, act);
-                if (lane == j) word = bits;
-            }
-            if (wi < w1) P.bitmap[wi] = word;
-        } else if (mode == F_UNCERT) {  // certificates: the uncertified queries' mask parks in M
-            for (uint32_t j = 0; j < 32; ++j) {
-                const uint32_t v = (g0 + j) * 32 + lane;
-                const uint32_t unc = (g0 + j < w1 && v < P.n) ? uncertified<KIND, L>(P, sh, nq, v) : 0u;
-                if (unc) P.M[v] = unc;
-                const uint32_t bits = __ballot_sync(FULL, unc != 0);
-                if (lane == j) word = bits;
-            }
-            if (wi < w1) P.bitmap[wi] = word;
-        } else if (mode == F_MASKS) {  // union frontier = {v : M[v] != 0}: all 32 loads in flight
-            uint32_t mv[32];
-#pragma unroll
-            for (uint32_t j = 0; j < 32; ++j) {
-                const uint32_t v = (g0 + j) * 32 + lane;
-                mv[j] = (g0 + j < w1 && v < P.n) ? ld_cg(P.M + v) : 0u;
-            }
-#pragma unroll
-            for (uint32_t j = 0; j < 32; ++j) {
-                const uint32_t bits = __ballot_sync(FULL, mv[j] != 0u);
-                if (lane == j) word = bits;
-            }
-            if (wi < w1) P.bitmap[wi] = word;
-        } else if (wi < w1) {
-            word = ld_cg(P.bitmap + wi);
-        }
+        if (wi < w1) word = ld_cg(P.bitmap + wi);
         active += __popc(word);
         uint32_t nz = __ballot_sync(FULL, word != 0);
         while (nz) {
@@ -389,12 +369,8 @@ __device__ void compact(const BParams& P, const GraphView& g, int mode, const ui
                 const uint32_t d = act ? deg[k] : 0u;
                 uint32_t mask = 0;
                 if (act) {
-                    if (mode == F_IMPACTED) {
-                        mask = row_live<L>(P.V, v);
-                    } else {
-                        mask = ld_cg(P.M + v);
-                        P.M[v] = 0u;  // consumed
-                    }
+                    mask = ld_cg(P.M + v);
+                    P.M[v] = 0u;  // consumed
                 }
                 uint32_t incl = d;
 #pragma unroll
@@ -413,6 +389,124 @@ __device__ void compact(const BParams& P, const GraphView& g, int mode, const ui
                 eb += __shfl_sync(FULL, incl, 31);
             }
         }
+    }
+}
+
+// S1 for large frontiers held as query masks M (F_MASKS, and F_IMPACTED / F_UNCERT after their
+// mark pass): no bitmap.  A warp takes 32 bitmap-word spans (1024 vertices) and issues the masks
+// and row offsets of 16 words (512 vertices) at once — one memory round trip per half instead of
+// a dependent degree fetch per active word.  Pass 1 counts and reserves the CTA's list range;
+// pass 2 re-reads (L2), writes the list and consumes the masks (deg-0 vertices included).
+__device__ __forceinline__ void span_loads(const BParams& P, const GraphView& g, uint32_t g0, uint32_t w1, int h,
+                                           uint32_t (&mv)[16], uint32_t (&dg)[16]) {
+    const uint32_t lane = threadIdx.x & 31;
+    uint32_t pv[16];
+#pragma unroll
+    for (int j = 0; j < 16; ++j) {
+        const uint32_t wj = g0 + h * 16 + j;
+        const uint32_t v = wj * 32 + lane;
+        const bool ok = wj < w1 && v < P.n;
+        mv[j] = ok ? ld_cg(P.M + v) : 0u;
+        pv[j] = __ldg(g.ptr + min(v, P.n));
+    }
+    const uint32_t pn = __ldg(g.ptr + min((g0 + h * 16 + 16) * 32, P.n));  // row offset after the span
+#pragma unroll
+    for (int j = 0; j < 16; ++j) {
+        uint32_t nx = __shfl_down_sync(FULL, pv[j], 1);
+        const uint32_t n31 = j < 15 ? __shfl_sync(FULL, pv[j < 15 ? j + 1 : j], 0) : pn;
+        if (lane == 31) nx = n31;
+        dg[j] = mv[j] ? nx - pv[j] : 0u;
+    }
+}
+
+__device__ void compact_masks(const BParams& P, const GraphView& g, unsigned long long* cnt_slot,
+                              unsigned long long* act_slot, uint32_t* sm) {
+    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint64_t W = P.words;
+    const uint32_t w0 = (uint32_t)(W * blockIdx.x / gridDim.x), w1 = (uint32_t)(W * (blockIdx.x + 1) / gridDim.x);
+    const uint32_t lt = (1u << lane) - 1u;
+    uint32_t cnt = 0, edges = 0, active = 0;
+    for (uint32_t g0 = w0 + warp * 32; g0 < w1; g0 += BW * 32)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            uint32_t mv[16], dg[16];
+            span_loads(P, g, g0, w1, h, mv, dg);
+#pragma unroll
+            for (int j = 0; j < 16; ++j) {
+                active += mv[j] != 0u;
+                cnt += dg[j] != 0u;
+                edges += dg[j];
+            }
+        }
+    for (int o = 16; o > 0; o >>= 1) {
+        cnt += __shfl_xor_sync(FULL, cnt, o);
+        edges += __shfl_xor_sync(FULL, edges, o);
+        active += __shfl_xor_sync(FULL, active, o);
+    }
+    if (lane == 0) {
+        sm[warp] = cnt;
+        sm[BW + warp] = edges;
+        if (active) atomicAdd(act_slot, (unsigned long long)active);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        uint32_t tc = 0, te = 0;
+        for (int i = 0; i < BW; ++i) {
+            const uint32_t c = sm[i], e = sm[BW + i];
+            sm[i] = tc;
+            sm[BW + i] = te;
+            tc += c;
+            te += e;
+        }
+        unsigned long long old = 0;
+        if (tc) old = atomicAdd(cnt_slot, ((unsigned long long)tc << 32) | te);
+        sm[2 * BW] = (uint32_t)(old >> 32);
+        sm[2 * BW + 1] = (uint32_t)old;
+    }
+    __syncthreads();
+    uint32_t pos = sm[2 * BW] + sm[warp];
+    uint32_t eb = sm[2 * BW + 1] + sm[BW + warp];
+    __syncthreads();
+    for (uint32_t g0 = w0 + warp * 32; g0 < w1; g0 += BW * 32)
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+            uint32_t mv[16], dg[16];
+            span_loads(P, g, g0, w1, h, mv, dg);
+#pragma unroll
+            for (int j = 0; j < 16; ++j) {
+                const uint32_t v = (g0 + h * 16 + j) * 32 + lane;
+                if (mv[j]) P.M[v] = 0u;  // consumed
+                const uint32_t d = dg[j];
+                uint32_t incl = d;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const uint32_t y = __shfl_up_sync(FULL, incl, o);
+                    if (lane >= (uint32_t)o) incl += y;
+                }
+                const uint32_t bal = __ballot_sync(FULL, d != 0);
+                if (d) {
+                    const uint32_t i = pos + __popc(bal & lt);
+                    P.lv[i] = v;
+                    P.lo[i] = eb + incl - d;
+                    P.lm[i] = mv[j];
+                }
+                pos += __popc(bal);
+                eb += __shfl_sync(FULL, incl, 31);
+            }
+        }
+}
+
+// Mark passes (thread per vertex, coalesced): F_IMPACTED — Alg 3 l.15, M[v] = the queries for
+// which Val(v) != InitVal; F_UNCERT — NEXT-1, M[v] = v's uncertified queries, only for vertices
+// with in-edges (the pull needs them).  M is all-zero before either.
+template <int KIND, class L>
+__device__ void mark_masks(const BParams& P, int mode, const uint32_t* sh, int nq) {
+    const uint64_t nth = (uint64_t)gridDim.x * BT;
+    for (uint64_t v = blockIdx.x * (uint64_t)BT + threadIdx.x; v < P.n; v += nth) {
+        uint32_t m;
+        if (mode == F_IMPACTED) m = row_live<L>(P.V, (uint32_t)v);
+        else m = __ldg(P.R.ptr + v + 1) > __ldg(P.R.ptr + v) ? uncertified<KIND, L>(P, sh, nq, (uint32_t)v) : 0u;
+        if (m) P.M[v] = m;
     }
 }
 
@@ -571,32 +665,74 @@ __device__ __forceinline__ uint32_t first_entry(const BParams& P, uint32_t count
 }
 
 // S2 over the compacted list: the iteration's E list edges split evenly over all warps; a warp
-// slides 32-entry windows (a hub row is shared by as many warps and CTAs as needed).
+// slides 32-entry windows (a hub row is shared by as many warps and CTAs as needed).  Windows
+// are prefetched one ahead: while window i's edges run, window i+1's source rows are already
+// being copied (cp.async) into the other half of xs and window i+2's list entries are loading.
 template <int KIND, bool PACKED, class L>
 __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, uint32_t E, uint32_t* xs, uint32_t* vs,
                         bool set_bits, bool fresh, uint32_t& n_edges, uint32_t& n_upd, uint32_t& n_read) {
+    constexpr int RW = L::RW;
+    using RC = RowCopy<L>;
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t gw = blockIdx.x * BW + (threadIdx.x >> 5);
     const uint64_t NW = (uint64_t)gridDim.x * BW;
     const uint32_t e0 = (uint32_t)((uint64_t)E * gw / NW), e1 = (uint32_t)((uint64_t)E * (gw + 1) / NW);
     if (e0 >= e1) return;
-    uint32_t i = first_entry(P, count, e0), e = e0;
-    for (;;) {
-        const uint32_t idx = i + lane;
-        uint32_t off = E, base = 0, v = 0, mask = 0;
+    auto list_load = [&](uint32_t i0, uint32_t& v, uint32_t& off, uint32_t& mask) {
+        const uint32_t idx = i0 + lane;
+        v = 0;
+        off = E;
+        mask = 0;
         if (idx < count) {
             v = ld_cg(P.lv + idx);
             off = ld_cg(P.lo + idx);
             mask = ld_cg(P.lm + idx);
-            base = __ldg(g.ptr + v) - off;
         }
-        load_rows<L>(P, xs, v, i, count);
-        const uint32_t wend = (i + 32 < count) ? ld_cg(P.lo + i + 32) : E;
+    };
+    auto rows_async = [&](uint32_t* buf, uint32_t v, uint32_t i0) {  // the window's 32 rows -> buf
+#pragma unroll
+        for (uint32_t r = 0; r < RC::C; ++r) {
+            const uint32_t f = r * 32 + lane, row = f / RC::C, c = f % RC::C;
+            const uint32_t vr = __shfl_sync(FULL, v, row);
+            if (i0 + row < count) RC::copy(buf + row * RW + c * RC::CW4, P.V + (size_t)vr * RW + c * RC::CW4, false);
+        }
+        cp_async_commit();
+    };
+    uint32_t i = first_entry(P, count, e0), e = e0;
+    uint32_t cv, coff, cmask, nv, noff, nmask;
+    list_load(i, cv, coff, cmask);
+    uint32_t cbase = i + lane < count ? __ldg(g.ptr + cv) - coff : 0u;
+    rows_async(xs, cv, i);
+    list_load(i + 32, nv, noff, nmask);
+    uint32_t buf = 0;
+    for (;;) {
+        const uint32_t wend = (i + 32 < count) ? __shfl_sync(FULL, noff, 0) : E;  // lo[i + 32]
         const uint32_t ehi = min(e1, wend);
-        window_edges<KIND, PACKED, L>(P, g, xs, vs, off, base, mask, e, ehi, set_bits, fresh, n_edges, n_upd, n_read);
-        if (ehi >= e1) break;
+        const bool more = ehi < e1;
+        uint32_t nbase = 0, mv = 0, moff = E, mmask = 0;
+        if (more) {
+            nbase = i + 32 + lane < count ? __ldg(g.ptr + nv) - noff : 0u;
+            rows_async(xs + (buf ^ 1) * 32 * RW, nv, i + 32);
+            list_load(i + 64, mv, moff, mmask);
+            cp_async_wait<1>();  // this window's rows (the next window's may still fly)
+        } else {
+            cp_async_wait<0>();
+        }
+        __syncwarp();
+        window_edges<KIND, PACKED, L>(P, g, xs + buf * 32 * RW, vs, coff, cbase, cmask, e, ehi, set_bits, fresh,
+                                      n_edges, n_upd, n_read);
+        __syncwarp();  // every lane is done with this window's rows before they are overwritten
+        if (!more) break;
         e = ehi;
         i += 32;
+        buf ^= 1;
+        cv = nv;
+        coff = noff;
+        cmask = nmask;
+        cbase = nbase;
+        nv = mv;
+        noff = moff;
+        nmask = mmask;
     }
 }
 
@@ -702,7 +838,9 @@ __device__ __forceinline__ uint32_t value_of(const uint32_t* V, uint32_t v, uint
     return L::decode(ld_cg(V + (size_t)v * L::RW + q / L::QPW), q % L::QPW);
 }
 
-// rows -> dst[(q0+q)*n + v] for q < nq, 32 vertices per warp through shared memory
+// rows -> dst[(q0+q)*n + v] for q < nq, 32 vertices per warp through shared memory: the 32
+// rows are read with 16 B loads (coalesced), each lane decodes its vertex's Q values, and every
+// query's 32 values leave as one 128 B streaming store
 template <class L>
 __device__ void transpose_out(const BParams& P, uint32_t* dst, int q0, int nq, uint32_t* xs) {
     constexpr int RW = L::RW;
@@ -711,22 +849,40 @@ __device__ void transpose_out(const BParams& P, uint32_t* dst, int q0, int nq, u
     const uint32_t NW = gridDim.x * BW;
     for (uint32_t v0 = gw * 32; v0 < P.n; v0 += NW * 32) {
         __syncwarp();
+        if constexpr (RW % 4 == 0) {
 #pragma unroll
-        for (int r = 0; r < RW; ++r) {
-            const uint32_t f = r * 32 + lane;
-            const uint32_t v = v0 + f / RW;
-            xs[(f / RW) * (RW + 1) + f % RW] = v < P.n ? ld_cg(P.V + (size_t)v * RW + f % RW) : 0u;
+            for (int r = 0; r < RW / 4; ++r) {
+                const uint32_t f = r * 32 + lane;  // 16 B chunk f of the 32 rows
+                const uint32_t v = v0 + f / (RW / 4), c = f % (RW / 4);
+                uint4 x = make_uint4(0, 0, 0, 0);
+                if (v < P.n)
+                    asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];"
+                                 : "=r"(x.x), "=r"(x.y), "=r"(x.z), "=r"(x.w)
+                                 : "l"(reinterpret_cast<const uint4*>(P.V + (size_t)v * RW) + c));
+                uint32_t* t = xs + (f / (RW / 4)) * (RW + 1) + 4 * c;
+                t[0] = x.x;
+                t[1] = x.y;
+                t[2] = x.z;
+                t[3] = x.w;
+            }
+        } else {
+#pragma unroll
+            for (int r = 0; r < RW; ++r) {
+                const uint32_t f = r * 32 + lane;
+                const uint32_t v = v0 + f / RW;
+                xs[(f / RW) * (RW + 1) + f % RW] = v < P.n ? ld_cg(P.V + (size_t)v * RW + f % RW) : 0u;
+            }
         }
         __syncwarp();
         const uint32_t v = v0 + lane;
         if (v < P.n)
             for (int q = 0; q < nq; ++q)
-                dst[(size_t)(q0 + q) * P.n + v] = L::decode(xs[lane * (RW + 1) + q / L::QPW], q % L::QPW);
+                __stcs(dst + (size_t)(q0 + q) * P.n + v, L::decode(xs[lane * (RW + 1) + q / L::QPW], q % L::QPW));
     }
 }
 
-template <class L>
-constexpr uint32_t xs_words() { return (32 * (L::RW + 1) + 3) & ~3u; }  // per warp, 16 B aligned
+template <class L>  // per warp, 16 B aligned: two 32-row windows (S2) or the padded transpose tile
+constexpr uint32_t xs_words() { return 2 * 32 * L::RW > ((32 * (L::RW + 1) + 3) & ~3u) ? 2 * 32 * L::RW : ((32 * (L::RW + 1) + 3) & ~3u); }
 template <class L>
 constexpr uint32_t vs_words() { return S_PIPE * 32 * L::RW; }
 
@@ -746,6 +902,9 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
     const uint64_t nthreads = (uint64_t)gridDim.x * BT;
     uint32_t ring = 0;
 
+    // kernel-level trace marks (tid 0): [cap-1] = {entry, seeds done, loop done, exit} of batch 0
+    unsigned long long* kt = (P.trace && tid == 0) ? P.trace + 5ull * (P.trace_cap - 1) : nullptr;
+    if (kt) kt[0] = global_ns();
     for (int q0 = 0; q0 < P.n_src; q0 += Q) {
         const int nq = min(Q, P.n_src - q0);
         // Alg 3 l.4, l.6 for every query of the batch; masks cleared
@@ -781,6 +940,7 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
             }
         }
         grid_sync(P.ctrl, epoch);
+        if (kt && q0 == 0) kt[1] = global_ns();
 
         int phase = P.two_phase ? 1 : 2;
         bool predicate = false;  // this iteration's S1 seeds Active with the impacted vertices
@@ -798,13 +958,21 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
             }
             const unsigned long long t_s0 = (P.trace && tid == 0) ? global_ns() : 0ull;
             const int mode = pull ? F_UNCERT : predicate ? F_IMPACTED : bits ? F_BITS : F_MASKS;
-            compact<KIND, L>(P, pull ? P.R : g, mode, sh, nq, ctr + CT_LIST, ctr + CT_ACTIVE, sm_cnt);
+            if (mode == F_BITS) {
+                compact_bits(P, g, ctr + CT_LIST, ctr + CT_ACTIVE, sm_cnt);
+            } else {
+                if (mode != F_MASKS) {  // impacted (l.15) / uncertified (NEXT-1) queries into M
+                    mark_masks<KIND, L>(P, mode, sh, nq);
+                    grid_sync(P.ctrl, epoch);
+                }
+                compact_masks(P, pull ? P.R : g, ctr + CT_LIST, ctr + CT_ACTIVE, sm_cnt);
+            }
             grid_sync(P.ctrl, epoch);
             ++ring;
             const unsigned long long ce = ld_cg64(ctr + CT_LIST);
             const uint32_t count = (uint32_t)(ce >> 32), E = (uint32_t)ce;
             const uint32_t tr = ring - 1;
-            if (P.trace && tid == 0 && tr < P.trace_cap) {
+            if (P.trace && tid == 0 && tr + 1 < P.trace_cap) {
                 unsigned long long* t = P.trace + 5ull * tr;
                 t[0] = t_s0;
                 t[1] = global_ns();
@@ -858,17 +1026,18 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
             } else {
                 // small frontier: its S2 sets frontier bits (few reds) and the next S1 reads the
                 // bitmap; large frontier: no bitmap reds (they contend in L2), the next S1 scans M
-                bits = count < P.bits_below;
+                bits = E < P.bits_below;  // at most E vertices change
                 relax_b<KIND, PACKED, L>(P, g, count, E, xs, vs, bits, fresh, n_edges, n_upd, n_read);
                 predicate = false;
             }
             grid_sync(P.ctrl, epoch);
-            if (P.trace && tid == 0 && tr < P.trace_cap) P.trace[5ull * tr + 2] = global_ns();
+            if (P.trace && tid == 0 && tr + 1 < P.trace_cap) P.trace[5ull * tr + 2] = global_ns();
             if (++iters > P.max_iters) {
                 if (tid == 0) atomicOr(P.err, ERR_ITERS);
                 return;
             }
         }
+        if (kt && q0 == 0) kt[2] = global_ns();
         transpose_out<L>(P, P.out, q0, nq, xs);
         if (P.stats) {  // reached / precise per query (the thread's query q is fixed)
             const uint32_t q = (uint32_t)(tid % Q);
@@ -888,6 +1057,7 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
         }
         grid_sync(P.ctrl, epoch);  // V / M / bitmap are reused by the next batch
     }
+    if (kt) kt[3] = global_ns();
 }
 
 template <int KIND, bool PACKED, int LW>
@@ -923,7 +1093,10 @@ void launch_kind_b(int kind, int lw, const BParams& P, int sms, cudaStream_t s) 
         if (lw == 16) launch_b<CG_SSNP, PACKED, 16>(P, sms, s);
         else launch_b<CG_SSNP, PACKED, 32>(P, sms, s);
         break;
-    case CG_VITERBI: launch_b<CG_VITERBI, PACKED, 32>(P, sms, s); break;
+    case CG_VITERBI:
+        if (lw == 33) launch_b<CG_VITERBI, PACKED, 33>(P, sms, s);
+        else launch_b<CG_VITERBI, PACKED, 32>(P, sms, s);
+        break;
     case CG_BFS:
         if (lw == 16) launch_b<CG_BFS, PACKED, 16>(P, sms, s);
         else launch_b<CG_BFS, PACKED, 32>(P, sms, s);
@@ -943,6 +1116,7 @@ int lane_width(const Graph& G, int kind) {
     const char* e = getenv("CG_LANES");
     if (e && atoi(e) == 32) return 32;
     if (kind == CG_REACH) return 1;
+    if (kind == CG_VITERBI) return (e && atoi(e) == 33) ? 33 : 32;  // CG_LANES=33: 32 per pass (measured slower)
     if (kind == CG_BFS) return 16;
     if ((kind == CG_SSSP || kind == CG_SSWP || kind == CG_SSNP) && G.w_max <= 2048) return 16;
     return 32;
@@ -953,7 +1127,7 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
     BatchSpace& w = G.bs;
     const uint32_t words = (G.n + 31) / 32;
     if (w.n != G.n) {
-        w.V.alloc((size_t)G.n * 16, s);  // the widest row: 16 u32 words
+        w.V.alloc((size_t)G.n * 32, s);  // the widest row: 32 u32 words (Viterbi, 32 per pass)
         w.M.alloc(G.n ? G.n : 1, s);
         w.bitmap.alloc(words ? words : 1, s);
         w.lv.alloc(G.n ? G.n : 1, s);
@@ -964,7 +1138,7 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
         w.n = G.n;
         w.B = 16;
     }
-    const int Q = lw == 32 ? 16 : 32;
+    const int Q = lw == 32 ? 16 : 32;  // (lw 33: u32 lanes, 32 per pass)
     DevBuf<unsigned long long> st;
     if (stats) st.alloc((size_t)c.n_src * NSTAT, s);
     BParams P{};
@@ -1033,7 +1207,12 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
         CGB_CUDA(cudaMemcpyAsync(h.data(), trace.get(), trace.bytes(), cudaMemcpyDeviceToHost, s));
         CGB_CUDA(cudaStreamSynchronize(s));
         unsigned long long t0 = 0;
-        for (uint32_t i = 0; i < P.trace_cap && h[5 * i]; ++i) {
+        {
+            const unsigned long long* k = h.data() + 5ull * (P.trace_cap - 1);
+            fprintf(stderr, "CG_TRACE_KERNEL kind=%d Q=%d lanes=%d init+seeds=%.1f batch0_loop_end=%.1f exit=%.1f us\n",
+                    c.kind, Q, lw, (k[1] - k[0]) / 1e3, (k[2] - k[0]) / 1e3, (k[3] - k[0]) / 1e3);
+        }
+        for (uint32_t i = 0; i < P.trace_cap - 1 && h[5 * i]; ++i) {
             const unsigned long long* t = h.data() + 5 * i;
             if (!t0) t0 = t[0];
             fprintf(stderr, "CG_TRACE kind=%d Q=%d lanes=%d it=%u q0=%llu phase=%llu list=%llu active=%llu edges=%llu "
@@ -1064,7 +1243,7 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
             o.scanned_p1 = (int64_t)x[ST_S1];
             o.scanned_p2 = (int64_t)x[ST_S2];
             o.batch_queries = Q;
-            o.row_bytes = lw == 1 ? 4 : 64;
+            o.row_bytes = lw == 1 ? 4 : lw == 33 ? 128 : 64;
         }
     }
 }

@@ -15,5 +15,5 @@ except Exception as e:
     print("bench failed", e, open(f"gpurun_out/{t}_bench.err").read()[-1500:])
 PY
 for k in ${KINDS:-sssp bfs}; do
-  CG_TRACE=1 timeout 120 python tools/profile_query.py --config c2 --kind $k --mode 2phase --batch 16 2> gpurun_out/${tag}_trace_${k}.txt >/dev/null
+  CG_TRACE=1 timeout 120 python tools/profile_query.py --config c2 --kind $k --mode 2phase --batch 32 --repeat 2 2> gpurun_out/${tag}_trace_${k}.txt > gpurun_out/${tag}_ev_${k}.txt
 done

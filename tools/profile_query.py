@@ -17,7 +17,7 @@ def main():
     p.add_argument("--config", default="c2")
     p.add_argument("--kind", default="sssp")
     p.add_argument("--mode", default="2phase")
-    p.add_argument("--batch", type=int, default=16)
+    p.add_argument("--batch", type=int, default=32)
     p.add_argument("--repeat", type=int, default=1)
     a = p.parse_args()
     import numpy as np
@@ -38,10 +38,14 @@ def main():
     g.query(a.kind, srcs, mode=a.mode, out=out)  # warm
     torch.cuda.synchronize()
     for _ in range(a.repeat):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         torch.cuda.nvtx.range_push("prof")
+        e0.record()
         g.query(a.kind, srcs, mode=a.mode, out=out)
+        e1.record()
         torch.cuda.nvtx.range_pop()
-    torch.cuda.synchronize()
+        torch.cuda.synchronize()
+        print(f"query {a.kind} {a.mode} batch={a.batch}: {e0.elapsed_time(e1):.3f} ms (events)", flush=True)
     print("done")
 
 
