@@ -134,6 +134,34 @@ cg_status cg_build(cg_graph g, cg_kind kind, int32_t K, cg_hub_policy policy, co
 cg_status cg_build_ex(cg_graph g, cg_kind kind, int32_t K, cg_hub_policy policy, const uint32_t* hubs,
                       uint64_t seed, cg_cg_alg alg, int32_t connectivity, void* stream);
 
+/*
+ * NEXT-4 sharded construction.  Algorithm 1 marks, for every hub, the tight
+ * edges of its forward and backward Identify queries and takes the union, so the
+ * hubs can be split across GPUs: cg_build_partial marks the flags of hubs [hub_begin, hub_end)
+ * of the K hubs `policy` selects (the same K on every rank) into `flags` (device, uint8[m], G's
+ * CSR order; zeroed first, no connectivity edges); the caller OR-reduces the ranks' flags
+ * (e.g. ncclAllReduce(ncclUint8, ncclMax)); cg_build_from_flags installs the merged flags as
+ * the kind's Core Graph, adding the connectivity edges (connectivity < 0: Alg 1's default, on)
+ * and compacting.  SSSP / SSWP / SSNP / Viterbi only: Algorithm 2 (BFS / REACH) labels
+ * vertices across hubs in order and is not split (CG_EUNSUPPORTED).  Merged
+ * builds keep no NEXT-1 hub certificates.  Both synchronise `stream`.
+ */
+cg_status cg_build_partial(cg_graph g, cg_kind kind, int32_t K, cg_hub_policy policy, const uint32_t* hubs,
+                           uint64_t seed, int32_t hub_begin, int32_t hub_end, uint8_t* flags, void* stream);
+cg_status cg_build_from_flags(cg_graph g, cg_kind kind, int32_t K, cg_hub_policy policy, const uint32_t* hubs,
+                              uint64_t seed, const uint8_t* flags, int32_t connectivity, void* stream);
+
+/*
+ * NEXT-4 persistence: the CG is identified once and used for all future queries.
+ * cg_core_save writes the kind's Core Graph (edge flags bit-packed in G's CSR order, hubs,
+ * algorithm, connectivity option) to the host file `path`; cg_core_load installs it for `kind`
+ * on a graph with the same n, m and canonical-CSR fingerprint (else CG_EINVAL), without the
+ * Identify queries.  CG_ENOCG (save before build), CG_EINVAL (I/O error, foreign or truncated
+ * file).  Both synchronise `stream`.
+ */
+cg_status cg_core_save(cg_graph g, cg_kind kind, const char* path, void* stream);
+cg_status cg_core_load(cg_graph g, cg_kind kind, const char* path, void* stream);
+
 /* Core Graph sizes for `kind`: m_cg edges, K hubs (hubs: host buffer of >= K entries, may be NULL),
  * build_ms = device time of the last cg_build for that kind.  CG_ENOCG if not built. */
 cg_status cg_core_info(cg_graph g, cg_kind kind, int64_t* m_cg, int32_t* K, uint32_t* hubs, float* build_ms);

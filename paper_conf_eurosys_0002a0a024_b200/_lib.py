@@ -39,7 +39,11 @@ class CGOverflow(CGError, OverflowError):
     pass
 
 
-_EXC = {-1: CGInvalid, -4: CGNoCoreGraph, -5: CGOverflow}
+class CGUnsupported(CGError):
+    pass
+
+
+_EXC = {-1: CGInvalid, -4: CGNoCoreGraph, -5: CGOverflow, -7: CGUnsupported}
 
 
 class Stats(ctypes.Structure):
@@ -74,6 +78,12 @@ _SIGS = {
     "cg_core_info": (ctypes.c_int, [_P, ctypes.c_int, ctypes.POINTER(ctypes.c_int64),
                                     ctypes.POINTER(ctypes.c_int32), _P, ctypes.POINTER(ctypes.c_float)]),
     "cg_core_export": (ctypes.c_int, [_P, ctypes.c_int, _P, _P]),
+    "cg_build_partial": (ctypes.c_int, [_P, ctypes.c_int, ctypes.c_int32, ctypes.c_int, _P, ctypes.c_uint64,
+                                        ctypes.c_int32, ctypes.c_int32, _P, _P]),
+    "cg_build_from_flags": (ctypes.c_int, [_P, ctypes.c_int, ctypes.c_int32, ctypes.c_int, _P, ctypes.c_uint64,
+                                           _P, ctypes.c_int32, _P]),
+    "cg_core_save": (ctypes.c_int, [_P, ctypes.c_int, ctypes.c_char_p, _P]),
+    "cg_core_load": (ctypes.c_int, [_P, ctypes.c_int, ctypes.c_char_p, _P]),
     "cg_query": (ctypes.c_int, [_P, ctypes.c_int, _P, ctypes.c_int32, ctypes.c_int, _P, _P, _P]),
     "cg_query_ex": (ctypes.c_int, [_P, ctypes.c_int, _P, ctypes.c_int32, ctypes.c_int, _P, _P, _P, _P]),
     "cg_query_host": (ctypes.c_int, [_P, ctypes.c_int, _P, ctypes.c_int32, ctypes.c_int, _P, ctypes.c_int32, _P]),

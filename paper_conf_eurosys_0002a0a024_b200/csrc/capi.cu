@@ -187,6 +187,44 @@ cg_status cg_build(cg_graph g, cg_kind kind, int32_t K, cg_hub_policy policy, co
     return cg_build_ex(g, kind, K, policy, hubs, seed, CG_ALG_AUTO, -1, stream);
 }
 
+cg_status cg_build_partial(cg_graph g, cg_kind kind, int32_t K, cg_hub_policy policy, const uint32_t* hubs,
+                           uint64_t seed, int32_t hub_begin, int32_t hub_end, uint8_t* flags, void* stream) {
+    return guard([&] {
+        CGB_CHECK(g != nullptr && (flags != nullptr || g->G.m == 0), CG_EINVAL, "null argument");
+        check_kind(kind);
+        CGB_CUDA(cudaSetDevice(g->G.device));
+        build_core_partial(g->G, kind, K, policy, hubs, seed, hub_begin, hub_end, flags, S(stream));
+    });
+}
+
+cg_status cg_build_from_flags(cg_graph g, cg_kind kind, int32_t K, cg_hub_policy policy, const uint32_t* hubs,
+                              uint64_t seed, const uint8_t* flags, int32_t connectivity, void* stream) {
+    return guard([&] {
+        CGB_CHECK(g != nullptr && (flags != nullptr || g->G.m == 0), CG_EINVAL, "null argument");
+        check_kind(kind);
+        CGB_CUDA(cudaSetDevice(g->G.device));
+        build_core_from_flags(g->G, kind, K, policy, hubs, seed, flags, connectivity, S(stream));
+    });
+}
+
+cg_status cg_core_save(cg_graph g, cg_kind kind, const char* path, void* stream) {
+    return guard([&] {
+        CGB_CHECK(g != nullptr && path != nullptr, CG_EINVAL, "null argument");
+        check_kind(kind);
+        CGB_CUDA(cudaSetDevice(g->G.device));
+        save_core(g->G, kind, path, S(stream));
+    });
+}
+
+cg_status cg_core_load(cg_graph g, cg_kind kind, const char* path, void* stream) {
+    return guard([&] {
+        CGB_CHECK(g != nullptr && path != nullptr, CG_EINVAL, "null argument");
+        check_kind(kind);
+        CGB_CUDA(cudaSetDevice(g->G.device));
+        load_core(g->G, kind, path, S(stream));
+    });
+}
+
 cg_status cg_core_info(cg_graph g, cg_kind kind, int64_t* m_cg, int32_t* K, uint32_t* hubs, float* build_ms) {
     return guard([&] {
         CGB_CHECK(g != nullptr, CG_EINVAL, "null graph");

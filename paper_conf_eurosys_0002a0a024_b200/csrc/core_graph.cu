@@ -17,6 +17,8 @@
 #include <cub/device/device_scan.cuh>
 
 #include <chrono>
+#include <cstdio>
+#include <string>
 #include <cstring>
 
 #include "graph.hpp"
@@ -404,37 +406,14 @@ void alg2(Graph& G, const std::vector<uint32_t>& hubs, uint8_t* flags, bool per_
 
 }  // namespace
 
-void build_core(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs_in, uint64_t seed, int alg,
-                int connectivity, cudaStream_t s) {
-    CGB_CHECK(kind >= 0 && kind <= CG_REACH, CG_EINVAL, "bad kind");
-    CGB_CHECK(K > 0 && (uint32_t)K <= G.n, CG_EINVAL, "K must be in [1, n]");
-    // reading Q9': the general CG keeps one Qid[] per traversal direction by default (DESIGN.md)
-    if (alg == CG_ALG_AUTO) alg = (kind == CG_BFS || kind == CG_REACH) ? CG_ALG_GENERAL_PERDIR : CG_ALG_SPECIALIZED;
-    CGB_CHECK(alg == CG_ALG_SPECIALIZED || alg == CG_ALG_GENERAL || alg == CG_ALG_GENERAL_PERDIR, CG_EINVAL,
-              "bad CG algorithm");
-    if (connectivity < 0) connectivity = (alg == CG_ALG_SPECIALIZED) ? 1 : 0;  // reading Q11
+namespace {
 
-    cudaEvent_t e0, e1;
-    CGB_CUDA(cudaEventCreate(&e0));
-    CGB_CUDA(cudaEventCreate(&e1));
-    CGB_CUDA(cudaEventRecord(e0, s));
-
-    std::vector<uint32_t> hubs = select_hubs(G, K, policy, hubs_in, seed, s);
-    Core& C = G.core[core_slot(kind)];
-    C.built = false;
-    C.hub_vals.reset();
-    C.hub_k = 0;
-    C.flags.alloc(G.m ? G.m : 1, s);
-    CGB_CUDA(cudaMemsetAsync(C.flags.get(), 0, C.flags.bytes(), s));
-    if (G.m) {
-        if (alg == CG_ALG_SPECIALIZED) alg1(G, kind, hubs, C.flags.get(), C, s);
-        else alg2(G, hubs, C.flags.get(), alg == CG_ALG_GENERAL_PERDIR, s);
-        if (connectivity) {
-            const int sel = (kind == CG_SSWP) ? 1 : ((kind == CG_BFS || kind == CG_REACH) ? 2 : 0);
-            CGB_LAUNCH(k_connectivity, grid_rows(G.n), TB, 0, s, G.n, view(G.g), G.dbits, sel, C.flags.get());
-        }
+// a6 + a7: connectivity edges (Alg 1 l.8-12) on C.flags, then stream compaction into C.adj
+void finalize_core(Graph& G, int kind, Core& C, int connectivity, cudaStream_t s) {
+    if (G.m && connectivity) {
+        const int sel = (kind == CG_SSWP) ? 1 : ((kind == CG_BFS || kind == CG_REACH) ? 2 : 0);
+        CGB_LAUNCH(k_connectivity, grid_rows(G.n), TB, 0, s, G.n, view(G.g), G.dbits, sel, C.flags.get());
     }
-    // a7: compaction into the CG's CSR
     DevBuf<uint32_t> cnt(G.n + 1, s);
     C.adj.n = G.n;
     C.adj.ptr.alloc(G.n + 1, s);
@@ -449,16 +428,205 @@ void build_core(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs_
     if (G.packed) C.adj.adj.alloc(adj_alloc_elems(mcg, 4), s); else C.adj.adjw.alloc(adj_alloc_elems(mcg, 8), s);
     CGB_LAUNCH(k_scatter_core, grid_rows(G.n), TB, 0, s, G.n, G.g.ptr.get(), C.flags.get(), C.adj.ptr.get(),
                G.g.adj.get(), G.g.adjw.get(), C.adj.adj.get(), C.adj.adjw.get());
-    CGB_CUDA(cudaEventRecord(e1, s));
-    CGB_CUDA(cudaEventSynchronize(e1));
-    float ms = 0.f;
-    CGB_CUDA(cudaEventElapsedTime(&ms, e0, e1));
-    cudaEventDestroy(e0);
-    cudaEventDestroy(e1);
+}
+
+struct Timer {
+    cudaEvent_t e0, e1;
+    cudaStream_t s;
+    explicit Timer(cudaStream_t st) : s(st) {
+        CGB_CUDA(cudaEventCreate(&e0));
+        CGB_CUDA(cudaEventCreate(&e1));
+        CGB_CUDA(cudaEventRecord(e0, s));
+    }
+    float stop() {
+        CGB_CUDA(cudaEventRecord(e1, s));
+        CGB_CUDA(cudaEventSynchronize(e1));
+        float ms = 0.f;
+        CGB_CUDA(cudaEventElapsedTime(&ms, e0, e1));
+        return ms;
+    }
+    ~Timer() {
+        cudaEventDestroy(e0);
+        cudaEventDestroy(e1);
+    }
+};
+
+bool alg1_kind(int kind) { return kind == CG_SSSP || kind == CG_SSWP || kind == CG_SSNP || kind == CG_VITERBI; }
+
+// order-independent 64-bit fingerprint of the canonical graph (row offsets and edge words)
+__device__ __forceinline__ unsigned long long mix64(unsigned long long x) {
+    x ^= x >> 30;
+    x *= 0xbf58476d1ce4e5b9ull;
+    x ^= x >> 27;
+    x *= 0x94d049bb133111ebull;
+    return x ^ (x >> 31);
+}
+__global__ void k_graph_hash(uint32_t n, uint32_t m, const uint32_t* __restrict__ ptr, const uint32_t* __restrict__ adj,
+                             const uint2* __restrict__ adjw, unsigned long long* out) {
+    unsigned long long h = 0;
+    const uint64_t tot = (uint64_t)n + 1 + m;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < tot; i += (uint64_t)gridDim.x * blockDim.x) {
+        unsigned long long x;
+        if (i <= n) x = ptr[i];
+        else if (adj) x = adj[i - n - 1];
+        else x = ((unsigned long long)adjw[i - n - 1].x << 32) | adjw[i - n - 1].y;
+        h += mix64(i * 0x9e3779b97f4a7c15ull ^ x);
+    }
+    for (int o = 16; o > 0; o >>= 1) h += __shfl_xor_sync(0xffffffffu, h, o);
+    if ((threadIdx.x & 31) == 0) atomicAdd(out, h);
+}
+
+unsigned long long graph_hash(Graph& G, cudaStream_t s) {
+    DevBuf<unsigned long long> d(1, s);
+    CGB_CUDA(cudaMemsetAsync(d.get(), 0, 8, s));
+    CGB_LAUNCH(k_graph_hash, 4 * G.num_sms, TB, 0, s, G.n, G.m, G.g.ptr.get(), G.g.adj.get(), G.g.adjw.get(), d.get());
+    unsigned long long h = 0;
+    CGB_CUDA(cudaMemcpyAsync(&h, d.get(), 8, cudaMemcpyDeviceToHost, s));
+    CGB_CUDA(cudaStreamSynchronize(s));
+    return h;
+}
+
+struct CoreFileHeader {  // cg_core_save / cg_core_load (little-endian)
+    char magic[8];       // "CGB200\0\1"
+    uint32_t version, kind, alg, connectivity, K, n, m, reserved;
+    unsigned long long graph_hash, m_cg;
+};
+const char kMagic[8] = {'C', 'G', 'B', '2', '0', '0', 0, 1};
+
+}  // namespace
+
+void build_core(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs_in, uint64_t seed, int alg,
+                int connectivity, cudaStream_t s) {
+    CGB_CHECK(kind >= 0 && kind <= CG_REACH, CG_EINVAL, "bad kind");
+    CGB_CHECK(K > 0 && (uint32_t)K <= G.n, CG_EINVAL, "K must be in [1, n]");
+    // reading Q9': the general CG keeps one Qid[] per traversal direction by default (DESIGN.md)
+    if (alg == CG_ALG_AUTO) alg = (kind == CG_BFS || kind == CG_REACH) ? CG_ALG_GENERAL_PERDIR : CG_ALG_SPECIALIZED;
+    CGB_CHECK(alg == CG_ALG_SPECIALIZED || alg == CG_ALG_GENERAL || alg == CG_ALG_GENERAL_PERDIR, CG_EINVAL,
+              "bad CG algorithm");
+    if (connectivity < 0) connectivity = (alg == CG_ALG_SPECIALIZED) ? 1 : 0;  // reading Q11
+
+    Timer t(s);
+    std::vector<uint32_t> hubs = select_hubs(G, K, policy, hubs_in, seed, s);
+    Core& C = G.core[core_slot(kind)];
+    C.built = false;
+    C.hub_vals.reset();
+    C.hub_k = 0;
+    C.flags.alloc(G.m ? G.m : 1, s);
+    CGB_CUDA(cudaMemsetAsync(C.flags.get(), 0, C.flags.bytes(), s));
+    if (G.m) {
+        if (alg == CG_ALG_SPECIALIZED) alg1(G, kind, hubs, C.flags.get(), C, s);
+        else alg2(G, hubs, C.flags.get(), alg == CG_ALG_GENERAL_PERDIR, s);
+    }
+    finalize_core(G, kind, C, connectivity, s);
     C.hubs = hubs;
     C.alg = alg;
     C.connectivity = connectivity;
-    C.build_ms = ms;
+    C.build_ms = t.stop();
+    C.built = true;
+}
+
+// NEXT-4: Algorithm 1 is a union over hubs (each hub's tight edges are marked independently,
+// P:757-786), so the 2K Identify queries can be split across GPUs: each rank marks the flags of
+// its hub range, the flags are OR-reduced (ncclAllReduce max on u8), and every rank finalises.
+// Algorithm 2 is sequential in the hubs (shared labels) and is not split.
+void build_core_partial(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs_in, uint64_t seed,
+                        int32_t hub_begin, int32_t hub_end, uint8_t* flags, cudaStream_t s) {
+    CGB_CHECK(alg1_kind(kind), CG_EUNSUPPORTED, "partial builds need Algorithm 1 (SSSP/SSWP/SSNP/Viterbi)");
+    CGB_CHECK(K > 0 && (uint32_t)K <= G.n, CG_EINVAL, "K must be in [1, n]");
+    CGB_CHECK(0 <= hub_begin && hub_begin <= hub_end && hub_end <= K, CG_EINVAL, "bad hub range");
+    std::vector<uint32_t> hubs = select_hubs(G, K, policy, hubs_in, seed, s);
+    if (G.m) CGB_CUDA(cudaMemsetAsync(flags, 0, G.m, s));
+    if (G.m && hub_end > hub_begin) {
+        std::vector<uint32_t> sub(hubs.begin() + hub_begin, hubs.begin() + hub_end);
+        Core scratch;  // no certificates are kept for partial builds
+        alg1(G, kind, sub, flags, scratch, s);
+    }
+    CGB_CUDA(cudaStreamSynchronize(s));
+}
+
+void build_core_from_flags(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs_in, uint64_t seed,
+                           const uint8_t* flags, int connectivity, cudaStream_t s) {
+    CGB_CHECK(alg1_kind(kind), CG_EUNSUPPORTED, "merged builds need Algorithm 1 (SSSP/SSWP/SSNP/Viterbi)");
+    CGB_CHECK(K > 0 && (uint32_t)K <= G.n, CG_EINVAL, "K must be in [1, n]");
+    if (connectivity < 0) connectivity = 1;  // reading Q11 for Algorithm 1
+    Timer t(s);
+    std::vector<uint32_t> hubs = select_hubs(G, K, policy, hubs_in, seed, s);
+    Core& C = G.core[core_slot(kind)];
+    C.built = false;
+    C.hub_vals.reset();
+    C.hub_k = 0;
+    C.flags.alloc(G.m ? G.m : 1, s);
+    if (G.m) CGB_CUDA(cudaMemcpyAsync(C.flags.get(), flags, G.m, cudaMemcpyDeviceToDevice, s));
+    finalize_core(G, kind, C, connectivity, s);
+    C.hubs = hubs;
+    C.alg = CG_ALG_SPECIALIZED;
+    C.connectivity = connectivity;
+    C.build_ms = t.stop();
+    C.built = true;
+}
+
+// NEXT-4 persistence: the CG is identified once for all future queries; the file
+// holds its edge flags (bit-packed, G's CSR order), hubs and options, tied to G by n, m and a
+// fingerprint of the canonical CSR.
+void save_core(Graph& G, int kind, const char* path, cudaStream_t s) {
+    const Core& C = G.core[core_slot(kind)];
+    CGB_CHECK(C.built, CG_ENOCG, "Core Graph not built for this kind");
+    std::vector<uint8_t> f(G.m);
+    if (G.m) CGB_CUDA(cudaMemcpyAsync(f.data(), C.flags.get(), G.m, cudaMemcpyDeviceToHost, s));
+    const unsigned long long h = graph_hash(G, s);
+    std::vector<uint8_t> bits((G.m + 7) / 8, 0);
+    for (size_t i = 0; i < f.size(); ++i)
+        if (f[i]) bits[i >> 3] |= (uint8_t)(1u << (i & 7));
+    CoreFileHeader hd{};
+    std::memcpy(hd.magic, kMagic, 8);
+    hd.version = 1;
+    hd.kind = (uint32_t)kind;
+    hd.alg = (uint32_t)C.alg;
+    hd.connectivity = (uint32_t)C.connectivity;
+    hd.K = (uint32_t)C.hubs.size();
+    hd.n = G.n;
+    hd.m = G.m;
+    hd.graph_hash = h;
+    hd.m_cg = C.adj.m;
+    FILE* fp = std::fopen(path, "wb");
+    CGB_CHECK(fp != nullptr, CG_EINVAL, std::string("cannot open for writing: ") + path);
+    bool ok = std::fwrite(&hd, sizeof hd, 1, fp) == 1;
+    ok = ok && (C.hubs.empty() || std::fwrite(C.hubs.data(), 4, C.hubs.size(), fp) == C.hubs.size());
+    ok = ok && (bits.empty() || std::fwrite(bits.data(), 1, bits.size(), fp) == bits.size());
+    ok = (std::fclose(fp) == 0) && ok;
+    CGB_CHECK(ok, CG_EINVAL, std::string("write failed: ") + path);
+}
+
+void load_core(Graph& G, int kind, const char* path, cudaStream_t s) {
+    FILE* fp = std::fopen(path, "rb");
+    CGB_CHECK(fp != nullptr, CG_EINVAL, std::string("cannot open: ") + path);
+    CoreFileHeader hd{};
+    bool ok = std::fread(&hd, sizeof hd, 1, fp) == 1 && std::memcmp(hd.magic, kMagic, 8) == 0 && hd.version == 1;
+    std::vector<uint32_t> hubs(ok ? hd.K : 0);
+    std::vector<uint8_t> bits(ok ? ((size_t)hd.m + 7) / 8 : 0);
+    ok = ok && (hubs.empty() || std::fread(hubs.data(), 4, hubs.size(), fp) == hubs.size());
+    ok = ok && (bits.empty() || std::fread(bits.data(), 1, bits.size(), fp) == bits.size());
+    std::fclose(fp);
+    CGB_CHECK(ok, CG_EINVAL, std::string("not a Core Graph file (or truncated): ") + path);
+    CGB_CHECK((int)hd.kind == kind || core_slot((int)hd.kind) == core_slot(kind), CG_EINVAL,
+              "the file holds the Core Graph of another kind");
+    CGB_CHECK(hd.n == G.n && hd.m == G.m && hd.graph_hash == graph_hash(G, s), CG_EINVAL,
+              "the file was saved for another graph (n, m or fingerprint differ)");
+    Timer t(s);
+    std::vector<uint8_t> f(G.m);
+    for (size_t i = 0; i < f.size(); ++i) f[i] = (bits[i >> 3] >> (i & 7)) & 1u;
+    Core& C = G.core[core_slot(kind)];
+    C.built = false;
+    C.hub_vals.reset();
+    C.hub_k = 0;
+    C.flags.alloc(G.m ? G.m : 1, s);
+    if (G.m) CGB_CUDA(cudaMemcpyAsync(C.flags.get(), f.data(), G.m, cudaMemcpyHostToDevice, s));
+    finalize_core(G, kind, C, 0, s);  // the saved flags already hold the connectivity edges
+    CGB_CHECK(C.adj.m == hd.m_cg, CG_EINVAL, "Core Graph file is inconsistent (edge count)");
+    C.hubs = hubs;
+    C.alg = (int)hd.alg;
+    C.connectivity = (int)hd.connectivity;
+    C.build_ms = t.stop();
     C.built = true;
 }
 

@@ -118,6 +118,12 @@ int batch_width();  // B of the batched engine (CG_BATCH env: 8 / 16 / 32; anyth
 void run_queries_batched(Graph& G, const QueryCall& c, int B, cudaStream_t s, std::vector<cg_stats>* stats);
 
 // core_graph.cu
+void build_core_partial(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs, uint64_t seed,
+                        int32_t hub_begin, int32_t hub_end, uint8_t* flags, cudaStream_t s);
+void build_core_from_flags(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs, uint64_t seed,
+                           const uint8_t* flags, int connectivity, cudaStream_t s);
+void save_core(Graph& G, int kind, const char* path, cudaStream_t s);
+void load_core(Graph& G, int kind, const char* path, cudaStream_t s);
 void build_core(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs, uint64_t seed, int alg,
                 int connectivity, cudaStream_t s);
 

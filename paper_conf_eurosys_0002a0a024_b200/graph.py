@@ -140,6 +140,52 @@ class Graph:
                       int(seed), CG_ALGS[alg], conn, _stream(self.device))
         return self.core_info(kind)
 
+    @staticmethod
+    def _hubs_arg(K, policy, hubs):
+        pol = HUB_POLICIES[policy]
+        harr = None
+        if hubs is not None:
+            pol = HUB_POLICIES["given"]
+            hl = [int(x) for x in hubs]
+            K = len(hl)
+            harr = (ctypes.c_uint32 * K)(*hl)
+        return K, pol, (ctypes.cast(harr, ctypes.c_void_p) if harr is not None else None), harr
+
+    def build_partial(self, kind, K: int = 20, hub_range=(0, None), policy: str = "topdeg", hubs=None,
+                      seed: int = 0) -> torch.Tensor:
+        """cg_build_partial (NEXT-4): Algorithm 1 edge flags (uint8[m], G's CSR order) of the hubs
+        hub_range = [begin, end) of the K hubs the policy selects."""
+        K, pol, hp, _keep = self._hubs_arg(K, policy, hubs)
+        b, e = hub_range
+        e = K if e is None else e
+        flags = torch.empty(max(self.m, 1), dtype=torch.uint8, device=self.device)
+        with torch.cuda.device(self.device):
+            _lib.call("cg_build_partial", self._h, kind_id(kind), int(K), pol, hp, int(seed), int(b), int(e),
+                      _ptr(flags), _stream(self.device))
+        return flags[:self.m]
+
+    def build_from_flags(self, kind, flags: torch.Tensor, K: int = 20, policy: str = "topdeg", hubs=None,
+                         seed: int = 0, connectivity: bool | None = None) -> dict:
+        """cg_build_from_flags (NEXT-4): install merged Algorithm 1 flags as the kind's CG."""
+        K, pol, hp, _keep = self._hubs_arg(K, policy, hubs)
+        flags = flags.to(self.device, torch.uint8).contiguous()
+        conn = -1 if connectivity is None else (1 if connectivity else 0)
+        with torch.cuda.device(self.device):
+            _lib.call("cg_build_from_flags", self._h, kind_id(kind), int(K), pol, hp, int(seed), _ptr(flags), conn,
+                      _stream(self.device))
+        return self.core_info(kind)
+
+    def save_core(self, kind, path: str) -> None:
+        """cg_core_save (NEXT-4): write the kind's Core Graph to a host file."""
+        with torch.cuda.device(self.device):
+            _lib.call("cg_core_save", self._h, kind_id(kind), str(path).encode(), _stream(self.device))
+
+    def load_core(self, kind, path: str) -> dict:
+        """cg_core_load (NEXT-4): install a saved Core Graph (same graph required)."""
+        with torch.cuda.device(self.device):
+            _lib.call("cg_core_load", self._h, kind_id(kind), str(path).encode(), _stream(self.device))
+        return self.core_info(kind)
+
     def core_info(self, kind) -> dict:
         m_cg, K, ms = ctypes.c_int64(), ctypes.c_int32(), ctypes.c_float()
         _lib.call("cg_core_info", self._h, kind_id(kind), ctypes.byref(m_cg), ctypes.byref(K), None,

@@ -40,3 +40,26 @@ def max_over_ranks(x: float, device=None) -> float:
     t = torch.tensor([x], dtype=torch.float64, device=device)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
+
+
+def hub_shard(K: int, rank: int, world: int) -> tuple[int, int]:
+    """[begin, end) of the hubs whose Identify queries rank runs in a sharded CG build (NEXT-4)."""
+    return shard(K, rank, world)
+
+
+def merge_flags(flags: torch.Tensor, group=None) -> torch.Tensor:
+    """OR of the ranks' Algorithm 1 edge flags (uint8 0/1): an all-reduce with MAX, in place
+    (ncclAllReduce(ncclUint8, ncclMax) over NVLink on GPUs; gloo in the CPU tests)."""
+    if dist.is_available() and dist.is_initialized() and dist.get_world_size(group) > 1:
+        dist.all_reduce(flags, op=dist.ReduceOp.MAX, group=group)
+    return flags
+
+
+def build_sharded(graph, kind, K: int = 20, rank: int = 0, world: int = 1, group=None, **kw) -> dict:
+    """Sharded Core Graph build (NEXT-4): every rank runs the Identify queries of
+    its hub shard (cg_build_partial), the flags are OR-reduced across ranks, and every rank
+    installs the same merged CG (cg_build_from_flags).  Algorithm 1 kinds only."""
+    b, e = hub_shard(K, rank, world)
+    flags = graph.build_partial(kind, K=K, hub_range=(b, e), **kw)
+    merge_flags(flags, group)
+    return graph.build_from_flags(kind, flags, K=K, **kw)

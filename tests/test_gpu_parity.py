@@ -357,3 +357,57 @@ def test_general_cg_per_direction():
         out = to_np(g.query(kind, to_dev(s), mode="2phase"))
         for i, x in enumerate(s):
             assert_values_equal(out[i], oracle.query(kind, og, int(x)), kind, "perdir")
+
+
+@pytest.mark.parametrize("kind", ["sssp", "sswp", "ssnp", "viterbi"])
+def test_partial_builds_merge_to_full_core_graph(kind):
+    """NEXT-4: the flags of hub shards (cg_build_partial), OR-ed and installed with
+    cg_build_from_flags, give exactly the single-call Core Graph (Algorithm 1 is a union over
+    hubs), and 2Phase queries on it match the oracle."""
+    n, m = 1 << 13, 16 << 13
+    src, dst, w = gen.rmat(n, m, w_max=29, seed=61)
+    g, og = both(n, src, dst, w)
+    ref = g.build(kind, K=20)
+    ref_flags = g.core_flags(kind).cpu().numpy()
+    merged = None
+    for b, e in ((0, 7), (7, 13), (13, 20)):
+        f = g.build_partial(kind, K=20, hub_range=(b, e))
+        merged = f.clone() if merged is None else torch.maximum(merged, f)
+    info = g.build_from_flags(kind, merged, K=20)
+    assert np.array_equal(g.core_flags(kind).cpu().numpy(), ref_flags)
+    assert info["m_cg"] == ref["m_cg"] and info["hubs"] == ref["hubs"]
+    sources = gen.sample_sources(n, src, dst, 9, seed=2)
+    out = to_np(g.query(kind, to_dev(sources), mode="2phase"))
+    for i, s in enumerate(sources):
+        assert_values_equal(out[i], oracle.query(kind, og, int(s)), kind, f"merged {kind} s={s}")
+    from paper_conf_eurosys_0002a0a024_b200 import CGUnsupported
+    with pytest.raises(CGUnsupported):
+        g.build_partial("reach", K=4, hub_range=(0, 2))
+
+
+def test_core_graph_save_load(tmp_path):
+    """NEXT-4 persistence: a saved Core Graph loads into a fresh Graph of the same edges (same
+    flags, hubs, results) and is refused by a different graph."""
+    from paper_conf_eurosys_0002a0a024_b200 import CGInvalid, Graph
+    n, m = 1 << 13, 16 << 13
+    src, dst, w = gen.rmat(n, m, w_max=29, seed=62)
+    g, og = both(n, src, dst, w)
+    sources = gen.sample_sources(n, src, dst, 7, seed=3)
+    for kind in ("sssp", "reach"):
+        info = g.build(kind, K=16)
+        path = str(tmp_path / f"{kind}.cg")
+        g.save_core(kind, path)
+        g2 = Graph(n, to_dev(src), to_dev(dst), to_dev(w))
+        info2 = g2.load_core(kind, path)
+        assert info2["m_cg"] == info["m_cg"] and info2["hubs"] == info["hubs"]
+        assert np.array_equal(g2.core_flags(kind).cpu().numpy(), g.core_flags(kind).cpu().numpy())
+        out = to_np(g2.query(kind, to_dev(sources), mode="2phase"))
+        for i, s in enumerate(sources):
+            assert_values_equal(out[i], oracle.query(kind, og, int(s)), kind, f"loaded {kind} s={s}")
+        g2.close()
+    src3, dst3, w3 = gen.rmat(n, m, w_max=29, seed=63)
+    g3 = Graph(n, to_dev(src3), to_dev(dst3), to_dev(w3))
+    with pytest.raises(CGInvalid):
+        g3.load_core("sssp", str(tmp_path / "sssp.cg"))
+    with pytest.raises(CGInvalid):
+        g3.load_core("sssp", str(tmp_path / "missing.cg"))

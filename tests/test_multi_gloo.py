@@ -73,3 +73,42 @@ def test_gather_world2(tmp_path):
     g = oracle.canonical_csr(n, src, dst, w)
     sources = gen.sample_sources(n, src, dst, 4, seed=5)
     assert np.array_equal(full, oracle.query_batch("sssp", g, sources))
+
+
+def _merge_worker(rank, world, port, out_path):
+    sys.path.insert(0, ROOT)
+    import gen
+    import oracle
+    from paper_conf_eurosys_0002a0a024_b200 import multi
+
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    n, K = 1 << 10, 12
+    src, dst, w = gen.rmat(n, 8 * n, w_max=31, seed=7)
+    g = oracle.canonical_csr(n, src, dst, w)
+    gr = oracle.transpose(g)
+    hubs = oracle.hubs_topdeg(g, gr, K)
+    b, e = multi.hub_shard(K, rank, world)
+    # this rank's Identify queries (the CPU oracle stands in for cg_build_partial on a GPU)
+    mine = torch.from_numpy(oracle.cg_alg1("sswp", g, gr, hubs[b:e], connectivity=False))
+    multi.merge_flags(mine)
+    if rank == 0:
+        np.save(out_path, mine.numpy())
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_sharded_core_graph_merge_world2(tmp_path):
+    """NEXT-4: Algorithm 1 is a union over hubs, so marking half the hubs per rank and OR-ing
+    the flags (all-reduce MAX over uint8) reproduces the single-process flags exactly."""
+    import gen
+    import oracle
+    out = str(tmp_path / "flags.npy")
+    mp.spawn(_merge_worker, args=(2, _free_port(), out), nprocs=2, join=True)
+    n, K = 1 << 10, 12
+    src, dst, w = gen.rmat(n, 8 * n, w_max=31, seed=7)
+    g = oracle.canonical_csr(n, src, dst, w)
+    gr = oracle.transpose(g)
+    exp = oracle.cg_alg1("sswp", g, gr, oracle.hubs_topdeg(g, gr, K), connectivity=False)
+    assert np.array_equal(np.load(out), exp)
