@@ -383,6 +383,30 @@ def main():
                 "peak_source": peak_src,
                 "alg_bytes_per_launch": tot_bytes / len(kinds)}
 
+    # ---- NEXT-3 WCC (a whole-graph query, reported beside the six-kind headline): 2Phase on
+    # REACH's general CG vs FULL, device-timed, same warm-up rule
+    wcc = None
+    if "reach" in build:
+        wout = torch.empty((1, cfg.n), dtype=torch.uint32, device=dev)
+        wms = {}
+        for mode in ("2phase", "full"):
+            for _ in range(args.warmup):
+                g.query("wcc", None, mode=mode, out=wout)
+            barrier()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            for _ in range(args.steps):
+                g.query("wcc", None, mode=mode, out=wout)
+            e1.record(stream)
+            barrier()
+            wms[mode] = multi.max_over_ranks(e0.elapsed_time(e1), dev) / args.steps
+        _, wp1, wst = g.query("wcc", None, mode="2phase", p1=True, stats=True)
+        n_comp = int(torch.unique(wout[0].to(torch.int64)).numel())
+        wcc = {"ms_2phase": wms["2phase"], "ms_full": wms["full"], "speedup": wms["full"] / wms["2phase"],
+               "components": n_comp, "iters_p1": wst[0]["iters_p1"], "iters_p2": wst[0]["iters_p2"],
+               "p1_precision_pct": 100.0 * wst[0]["precise_p1"] / max(1, wst[0]["reached"])}
+        del wp1
+
     # ---- e2e through the public API with HOST buffers (pinned), copies inside the timed region
     e2e = None
     if not args.no_e2e:
@@ -424,7 +448,7 @@ def main():
                        "parallelism": f"source-sharded x{ws}, graph replicated", "gather": gather},
             "gteps": gteps2, "full": {"value": qpsf, "unit": "queries/s", "gteps": gtepsf, "ms_per_step": msf / args.steps},
             "speedup_2phase_vs_full": qpsf and qps2 / qpsf,
-            "per_kind": per_kind, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
+            "per_kind": per_kind, "wcc": wcc, "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e,
             "gpu_launches": launches, "clocks": clocks,
             "build_ms": {k: build[k]["build_ms"] for k in build}, "graph_build_s": graph_s,
         }

@@ -48,7 +48,14 @@ typedef enum {
 /* The six query kinds (north_star; Table 6 P:1496-1535 for SSSP/SSWP/SSNP/Viterbi/REACH;
  * BFS = hop count, reading D1).  Value words are u32 for all kinds except
  * VITERBI, whose value is an IEEE binary32 probability stored in the same 32-bit slot. */
-typedef enum { CG_SSSP = 0, CG_SSWP = 1, CG_SSNP = 2, CG_VITERBI = 3, CG_BFS = 4, CG_REACH = 5 } cg_kind;
+typedef enum { CG_SSSP = 0, CG_SSWP = 1, CG_SSNP = 2, CG_VITERBI = 3, CG_BFS = 4, CG_REACH = 5, CG_WCC = 6 } cg_kind;
+/* CG_WCC (Table 6 WCC row P:1532-1535): weakly connected
+ * components by label propagation — Val(v) starts at v for every vertex, all vertices active,
+ * Needed Val(v) > Val(u), EdgeFunction CASMIN(Val(v), Val(u)), over BOTH edge directions; the
+ * fixpoint is the minimum vertex id of v's weakly connected component.  It is a whole-graph
+ * query: cg_query takes n_src == 1 (src may be NULL) and writes n labels.  2PHASE runs phase 1
+ * on the general Core Graph (Alg 2, shared with BFS / REACH) and phase 2 on G from every
+ * vertex (reading W2). */
 
 /* CG_MODE_2PHASE: Algorithm 3 — phase 1 on the Core Graph, phase 2 on G
  * from the impacted set.  CG_MODE_FULL: the baseline, the same relaxation on G only. */

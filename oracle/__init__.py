@@ -32,7 +32,7 @@ _SRC = os.path.join(_HERE, "oracle.c")
 _LIB = os.path.join(_HERE, "liboracle.so")
 _lib = None
 
-KINDS = {"sssp": 0, "sswp": 1, "ssnp": 2, "viterbi": 3, "bfs": 4, "reach": 5}
+KINDS = {"sssp": 0, "sswp": 1, "ssnp": 2, "viterbi": 3, "bfs": 4, "reach": 5, "wcc": 6}
 KIND_NAMES = {v: k for k, v in KINDS.items()}
 
 
@@ -76,6 +76,7 @@ def _load():
         "or_subgraph": (i64, [i64, P, P, P, P, P, P, P]),
         "or_2phase": (None, [c_int, i64, P, P, P, P, P, P, u32, P, P, ctypes.POINTER(_Stats)]),
         "or_full_bsp": (None, [c_int, i64, P, P, P, u32, P, ctypes.POINTER(_Stats)]),
+        "or_wcc": (None, [i64, P, P, P]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -144,8 +145,18 @@ def _nz(a: np.ndarray) -> np.ndarray:
 
 
 def query(kind, g: CSR, s: int) -> np.ndarray:
+    if kind == "wcc" or kind == 6:
+        return wcc(g)  # a whole-graph query: the source is ignored
     out = np.empty(g.n, dtype=np.uint32)
     _load().or_query(_kind(kind), g.n, _p(g.ptr), _p(_nz(g.col)), _p(_nz(g.wt)), int(s), _p(out))
+    return out
+
+
+def wcc(g: CSR) -> np.ndarray:
+    """WCC labels (NEXT-3): the minimum vertex id of each vertex's weakly connected component
+    (the fixpoint of Table 6's WCC row), by union-find over the undirected edges."""
+    out = np.empty(g.n, dtype=np.uint32)
+    _load().or_wcc(g.n, _p(g.ptr), _p(_nz(g.col)), _p(out))
     return out
 
 

@@ -31,6 +31,8 @@
  *    shared Qid[] (readings Q9-Q11).
  *  - or_2phase / or_full_bsp: Algorithm 3 literally in
  *    sequential BSP order (readings Q1-Q5).
+ *  - or_wcc: weakly connected components (NEXT-3, Table 6 WCC row): the
+ *    minimum vertex id of each weak component, by union-find.
  *
  * Value words: every kind stores a 32-bit word per vertex; Viterbi stores
  * the IEEE-754 binary32 bit pattern (reading Q13: f32, RN division).
@@ -586,4 +588,30 @@ void or_full_bsp(int kind, int64_t n, const int64_t* ptr, const uint32_t* col, c
     if (st) *st = z;
     free(act);
     free(nxt);
+}
+
+/* ---------------------------------------------------------------- WCC (NEXT-3)
+ * Weakly connected components, the fixpoint of Table 6's WCC row: label
+ * propagation from Val(v) = v with CASMIN over both edge directions converges to the minimum
+ * vertex id of v's weakly connected component.  The oracle computes that definition directly:
+ * union-find over the undirected edges, then the smallest id of every set. */
+static int64_t uf_find(int64_t* par, int64_t x) {
+    while (par[x] != x) {
+        par[x] = par[par[x]];
+        x = par[x];
+    }
+    return x;
+}
+
+void or_wcc(int64_t n, const int64_t* ptr, const uint32_t* col, uint32_t* out) {
+    int64_t* par = (int64_t*)malloc(sizeof(int64_t) * (size_t)(n > 0 ? n : 1));
+    for (int64_t v = 0; v < n; ++v) par[v] = v;
+    for (int64_t u = 0; u < n; ++u)
+        for (int64_t e = ptr[u]; e < ptr[u + 1]; ++e) {
+            int64_t a = uf_find(par, u), b = uf_find(par, (int64_t)col[e]);
+            if (a == b) continue;
+            if (a < b) par[b] = a; else par[a] = b; /* the root is the smaller id */
+        }
+    for (int64_t v = 0; v < n; ++v) out[v] = (uint32_t)uf_find(par, v);
+    free(par);
 }

@@ -77,7 +77,7 @@ cg_status guard(F&& f) {
 
 inline cudaStream_t S(void* s) { return (cudaStream_t)s; }
 
-void check_kind(int kind) { CGB_CHECK(kind >= CG_SSSP && kind <= CG_REACH, CG_EINVAL, "bad cg_kind"); }
+void check_kind(int kind) { CGB_CHECK(kind >= CG_SSSP && kind <= CG_WCC, CG_EINVAL, "bad cg_kind"); }
 
 void check_sources_host(const Graph& G, const uint32_t* src, int32_t n_src) {
     for (int32_t i = 0; i < n_src; ++i) CGB_CHECK(src[i] < G.n, CG_EINVAL, "source id >= n");
@@ -93,7 +93,8 @@ void prepare_query(cg_graph g, int kind, int32_t n_src, int mode, const void* ou
     check_kind(kind);
     CGB_CHECK(n_src >= 0, CG_EINVAL, "n_src < 0");
     CGB_CHECK(mode == CG_MODE_2PHASE || mode == CG_MODE_FULL, CG_EINVAL, "bad cg_mode");
-    CGB_CHECK(n_src == 0 || (out && src), CG_EINVAL, "null src/out");
+    CGB_CHECK(n_src == 0 || (out && (src || kind == CG_WCC)), CG_EINVAL, "null src/out");
+    CGB_CHECK(kind != CG_WCC || n_src <= 1, CG_EINVAL, "CG_WCC is a whole-graph query: n_src must be 1");
     if (kind == CG_SSSP)
         CGB_CHECK((uint64_t)(g->G.n - 1) * g->G.w_max < 0xFFFFFFFFull, CG_EOVERFLOW,
                   "(n-1)*w_max >= 2^32-1: SSSP distances could wrap");
@@ -257,7 +258,9 @@ cg_status cg_query_ex(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_s
         if (n_src == 0) return;
         Graph& G = g->G;
         CGB_CUDA(cudaSetDevice(G.device));
-        if (stats) {  // validate sources on device (the call synchronises anyway)
+        if (kind == CG_WCC) src = nullptr;  // whole-graph query: no source
+        if (kind == CG_WCC) ensure_wcc_graphs(G, mode == CG_MODE_2PHASE, S(stream));
+        if (stats && src) {  // validate sources on device (the call synchronises anyway)
             DevBuf<uint32_t> bad(1, S(stream));
             CGB_CUDA(cudaMemsetAsync(bad.get(), 0, 4, S(stream)));
             CGB_LAUNCH(k_check_src, 1, 256, 0, S(stream), src, n_src, G.n, bad.get());
@@ -267,7 +270,9 @@ cg_status cg_query_ex(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_s
             CGB_CHECK(!hb, CG_EINVAL, "source id >= n");
         }
         const bool two = mode == CG_MODE_2PHASE;
-        QueryCall c{(int)kind, &G.g, two ? &G.core[core_slot(kind)].adj : &G.g, two ? 1 : 0, src, n_src,
+        Adj* full = kind == CG_WCC ? &G.gsym : &G.g;
+        Adj* core = kind == CG_WCC ? &G.core[CG_REACH].sym : &G.core[core_slot(kind)].adj;
+        QueryCall c{(int)kind, full, two ? core : full, two ? 1 : 0, src, n_src,
                     (uint32_t*)out, two ? (uint32_t*)p1_out : nullptr, stats != nullptr};
         std::vector<cg_stats> st;
         run_queries(G, c, S(stream), stats ? &st : nullptr);
@@ -286,9 +291,11 @@ cg_status cg_query_host(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n
         prepare_query(g, kind, n_src, mode, out, src);
         if (n_src == 0) return;
         Graph& G = g->G;
-        check_sources_host(G, src, n_src);
+        if (kind == CG_WCC) src = nullptr;
+        if (src) check_sources_host(G, src, n_src);
         CGB_CUDA(cudaSetDevice(G.device));
         cudaStream_t s = S(stream);
+        if (kind == CG_WCC) ensure_wcc_graphs(G, mode == CG_MODE_2PHASE, s);
         const size_t row = (size_t)G.n * 4;
         if (batch <= 0) {  // ~256 MiB of results per batch, at least 1 query
             size_t b = ((size_t)256 << 20) / (row ? row : 1);
@@ -296,7 +303,7 @@ cg_status cg_query_host(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n
         }
         if (batch > n_src) batch = n_src;
         DevBuf<uint32_t> dsrc((size_t)n_src, s);
-        CGB_CUDA(cudaMemcpyAsync(dsrc.get(), src, 4ull * n_src, cudaMemcpyHostToDevice, s));
+        if (src) CGB_CUDA(cudaMemcpyAsync(dsrc.get(), src, 4ull * n_src, cudaMemcpyHostToDevice, s));
         // two result slots: batch b computes on `s` into slot b%2 while batch b-1 drains on `cp`
         DevBuf<uint32_t> slot[2];
         slot[0].alloc((size_t)batch * G.n, s);
@@ -314,7 +321,9 @@ cg_status cg_query_host(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n
             const int32_t nq = (n_src - q0) < batch ? (n_src - q0) : batch;
             const int k = b & 1;
             if (b >= 2) CGB_CUDA(cudaStreamWaitEvent(s, drained[k], 0));
-            QueryCall c{(int)kind, &G.g, two ? &G.core[core_slot(kind)].adj : &G.g, two ? 1 : 0, dsrc.get() + q0,
+            Adj* full = kind == CG_WCC ? &G.gsym : &G.g;
+            Adj* core = kind == CG_WCC ? &G.core[CG_REACH].sym : &G.core[core_slot(kind)].adj;
+            QueryCall c{(int)kind, full, two ? core : full, two ? 1 : 0, src ? dsrc.get() + q0 : nullptr,
                         nq, slot[k].get(), nullptr, false};
             run_queries(G, c, s, nullptr);
             CGB_CUDA(cudaEventRecord(done[k], s));

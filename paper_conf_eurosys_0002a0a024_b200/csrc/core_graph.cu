@@ -497,8 +497,9 @@ const char kMagic[8] = {'C', 'G', 'B', '2', '0', '0', 0, 1};
 
 void build_core(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs_in, uint64_t seed, int alg,
                 int connectivity, cudaStream_t s) {
-    CGB_CHECK(kind >= 0 && kind <= CG_REACH, CG_EINVAL, "bad kind");
+    CGB_CHECK(kind >= 0 && kind <= CG_WCC, CG_EINVAL, "bad kind");
     CGB_CHECK(K > 0 && (uint32_t)K <= G.n, CG_EINVAL, "K must be in [1, n]");
+    if (kind == CG_WCC) kind = CG_REACH;  // WCC uses REACH's general CG; its G ∪ G^R is made per query
     // reading Q9': the general CG keeps one Qid[] per traversal direction by default
     if (alg == CG_ALG_AUTO) alg = (kind == CG_BFS || kind == CG_REACH) ? CG_ALG_GENERAL_PERDIR : CG_ALG_SPECIALIZED;
     CGB_CHECK(alg == CG_ALG_SPECIALIZED || alg == CG_ALG_GENERAL || alg == CG_ALG_GENERAL_PERDIR, CG_EINVAL,
@@ -509,6 +510,7 @@ void build_core(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs_
     std::vector<uint32_t> hubs = select_hubs(G, K, policy, hubs_in, seed, s);
     Core& C = G.core[core_slot(kind)];
     C.built = false;
+    C.sym_built = false;
     C.hub_vals.reset();
     C.hub_k = 0;
     C.flags.alloc(G.m ? G.m : 1, s);
@@ -523,6 +525,91 @@ void build_core(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs_
     C.connectivity = connectivity;
     C.build_ms = t.stop();
     C.built = true;
+}
+
+// ------------------------------------------------------------------ WCC graphs (NEXT-3)
+// Row v of the symmetrised graph = v's (flagged) out-edges in G followed by its (flagged)
+// in-edges (G^R row v; an in-edge's flag is that of its CSR edge, reid).  Edge words keep G's
+// encoding (the WCC EdgeFunction ignores the weight).
+__global__ void k_sym_count(uint32_t n, const uint32_t* __restrict__ gp, const uint32_t* __restrict__ rp,
+                            const uint32_t* __restrict__ reid, const uint8_t* __restrict__ flags,
+                            uint32_t* __restrict__ cnt) {
+    const uint32_t lane = threadIdx.x & 31;
+    const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
+    for (uint64_t u = blockIdx.x * (uint64_t)(blockDim.x / 32) + (threadIdx.x >> 5); u <= n; u += nw) {
+        if (u == n) { if (lane == 0) cnt[n] = 0; continue; }
+        uint32_t c = 0;
+        if (flags) {
+            for (uint32_t e = gp[u] + lane; e < gp[u + 1]; e += 32) c += flags[e] != 0;
+            for (uint32_t e = rp[u] + lane; e < rp[u + 1]; e += 32) c += flags[reid[e]] != 0;
+            for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(FULLM, c, o);
+        } else {
+            c = (gp[u + 1] - gp[u]) + (rp[u + 1] - rp[u]);
+        }
+        if (lane == 0) cnt[u] = c;
+    }
+}
+
+__device__ __forceinline__ void sym_copy_row(uint32_t r0, uint32_t r1, const uint32_t* __restrict__ reid,
+                                             const uint8_t* __restrict__ flags, const uint32_t* __restrict__ adj,
+                                             const uint2* __restrict__ adjw, uint32_t* __restrict__ sadj,
+                                             uint2* __restrict__ sadjw, uint32_t& o) {
+    const uint32_t lane = threadIdx.x & 31;
+    for (uint32_t b = r0; b < r1; b += 32) {
+        const uint32_t e = b + lane;
+        const bool f = e < r1 && (!flags || flags[reid ? reid[e] : e]);
+        const uint32_t bal = __ballot_sync(FULLM, f);
+        if (f) {
+            const uint32_t p = o + __popc(bal & ((1u << lane) - 1u));
+            if (adj) sadj[p] = adj[e]; else sadjw[p] = adjw[e];
+        }
+        o += __popc(bal);
+    }
+}
+
+__global__ void k_sym_scatter(uint32_t n, const uint32_t* __restrict__ gp, const uint32_t* __restrict__ rp,
+                              const uint32_t* __restrict__ reid, const uint8_t* __restrict__ flags,
+                              const uint32_t* __restrict__ sp, const uint32_t* __restrict__ gadj,
+                              const uint2* __restrict__ gadjw, const uint32_t* __restrict__ radj,
+                              const uint2* __restrict__ radjw, uint32_t* __restrict__ sadj, uint2* __restrict__ sadjw) {
+    const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
+    for (uint64_t u = blockIdx.x * (uint64_t)(blockDim.x / 32) + (threadIdx.x >> 5); u < n; u += nw) {
+        uint32_t o = sp[u];
+        sym_copy_row(gp[u], gp[u + 1], nullptr, flags, gadj, gadjw, sadj, sadjw, o);
+        sym_copy_row(rp[u], rp[u + 1], reid, flags, radj, radjw, sadj, sadjw, o);
+    }
+}
+
+void symmetrize(Graph& G, const uint8_t* flags, Adj& out, cudaStream_t s) {
+    DevBuf<uint32_t> cnt(G.n + 1, s);
+    CGB_LAUNCH(k_sym_count, grid_rows(G.n + 1), TB, 0, s, G.n, G.g.ptr.get(), G.gr.ptr.get(), G.reid.get(), flags,
+               cnt.get());
+    out.n = G.n;
+    out.ptr.alloc(G.n + 1, s);
+    exclusive_sum(cnt.get(), out.ptr.get(), (uint64_t)G.n + 1, s);
+    uint32_t ms = 0;
+    CGB_CUDA(cudaMemcpyAsync(&ms, out.ptr.get() + G.n, 4, cudaMemcpyDeviceToHost, s));
+    CGB_CUDA(cudaStreamSynchronize(s));
+    out.m = ms;
+    out.adj.reset();
+    out.adjw.reset();
+    if (G.packed) out.adj.alloc(adj_alloc_elems(ms, 4), s); else out.adjw.alloc(adj_alloc_elems(ms, 8), s);
+    CGB_LAUNCH(k_sym_scatter, grid_rows(G.n), TB, 0, s, G.n, G.g.ptr.get(), G.gr.ptr.get(), G.reid.get(), flags,
+               out.ptr.get(), G.g.adj.get(), G.g.adjw.get(), G.gr.adj.get(), G.gr.adjw.get(), out.adj.get(),
+               out.adjw.get());
+    CGB_CUDA(cudaStreamSynchronize(s));
+}
+
+void ensure_wcc_graphs(Graph& G, bool two_phase, cudaStream_t s) {
+    if (!G.gsym_built) {
+        symmetrize(G, nullptr, G.gsym, s);
+        G.gsym_built = true;
+    }
+    Core& C = G.core[CG_REACH];
+    if (two_phase && C.built && !C.sym_built) {
+        symmetrize(G, C.flags.get(), C.sym, s);
+        C.sym_built = true;
+    }
 }
 
 // NEXT-4: Algorithm 1 is a union over hubs (each hub's tight edges are marked independently,
@@ -553,6 +640,7 @@ void build_core_from_flags(Graph& G, int kind, int32_t K, int policy, const uint
     std::vector<uint32_t> hubs = select_hubs(G, K, policy, hubs_in, seed, s);
     Core& C = G.core[core_slot(kind)];
     C.built = false;
+    C.sym_built = false;
     C.hub_vals.reset();
     C.hub_k = 0;
     C.flags.alloc(G.m ? G.m : 1, s);
@@ -617,6 +705,7 @@ void load_core(Graph& G, int kind, const char* path, cudaStream_t s) {
     for (size_t i = 0; i < f.size(); ++i) f[i] = (bits[i >> 3] >> (i & 7)) & 1u;
     Core& C = G.core[core_slot(kind)];
     C.built = false;
+    C.sym_built = false;
     C.hub_vals.reset();
     C.hub_k = 0;
     C.flags.alloc(G.m ? G.m : 1, s);

@@ -191,7 +191,42 @@ struct LanesBit {
     }
 };
 
+// WCC (NEXT-3; Table 6 WCC row): one label per vertex, Val(v) = v initially, every vertex
+// active at the start of both phases (reading W2), cand = Val(u), select min (red.min).
+struct LanesLabel {
+    static constexpr int Q = 1, QPW = 1, RW = 1, G = 1;
+    static constexpr bool ALL_ACTIVE = true;
+    __device__ static uint32_t init_word() { return 0xffffffffu; }  // (never a label: the stats' "unreached")
+    __device__ static uint32_t init_at(uint64_t i) { return (uint32_t)i; }
+    __device__ static uint32_t decode(uint32_t x, uint32_t) { return x; }
+    __device__ static uint32_t live(uint32_t) { return 1u; }
+    __device__ static uint32_t top(uint32_t) { return 0u; }
+    __device__ static void seed(uint32_t*, uint32_t, uint32_t) {}
+    __device__ static uint32_t src_val() { return 0u; }
+    __device__ static uint32_t nb_val(uint32_t) { return 0u; }
+    __device__ static uint32_t relax(uint32_t* p, const uint32_t (&u)[G], const uint32_t (&c)[G], uint32_t,
+                                     uint32_t act, uint32_t& n_edges, uint32_t& n_upd, uint32_t*) {
+        if (!act) return 0u;
+        ++n_edges;
+        if (u[0] >= c[0]) return 0u;  // Needed: Val(v) > Val(u)
+        red_min(p, u[0]);             // CASMIN(Val(v), Val(u))
+        ++n_upd;
+        return 1u;
+    }
+};
+
+// per-vertex initial word and "every vertex starts active" for the policies that need them
+template <class L, class = void> struct InitOf {
+    static constexpr bool ALL_ACTIVE = false;
+    __device__ static uint32_t at(uint64_t) { return L::init_word(); }
+};
+template <class L> struct InitOf<L, decltype((void)L::ALL_ACTIVE, void())> {
+    static constexpr bool ALL_ACTIVE = L::ALL_ACTIVE;
+    __device__ static uint32_t at(uint64_t i) { return L::init_at(i); }
+};
+
 template <int LW, int KIND> struct LanesOf;
+template <int KIND> struct LanesOf<2, KIND> { using T = LanesLabel; };
 template <int KIND> struct LanesOf<32, KIND> { using T = Lanes32<KIND, 16>; };  // u32 fallback: 16 per pass
 template <int KIND> struct LanesOf<33, KIND> { using T = Lanes32<KIND, 32>; };  // Viterbi: 32 per pass (128 B rows)
 template <int KIND> struct LanesOf<16, KIND> { using T = Lanes16<KIND>; };
@@ -908,10 +943,10 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
     for (int q0 = 0; q0 < P.n_src; q0 += Q) {
         const int nq = min(Q, P.n_src - q0);
         // Alg 3 l.4, l.6 for every query of the batch; masks cleared
-        for (uint64_t i = tid; i < (uint64_t)P.n * RW; i += nthreads) P.V[i] = L::init_word();
-        for (uint64_t v = tid; v < P.n; v += nthreads) P.M[v] = 0u;
+        for (uint64_t i = tid; i < (uint64_t)P.n * RW; i += nthreads) P.V[i] = InitOf<L>::at(i);
+        for (uint64_t v = tid; v < P.n; v += nthreads) P.M[v] = InitOf<L>::ALL_ACTIVE ? 1u : 0u;
         grid_sync(P.ctrl, epoch);
-        for (int b = 0; b < nq; ++b) {
+        for (int b = 0; b < nq && !InitOf<L>::ALL_ACTIVE; ++b) {
             const uint32_t s = __ldg(P.srcs + q0 + b);
             if (s >= P.n) {
                 if (tid == 0) atomicOr(P.err, ERR_SOURCE);
@@ -944,7 +979,7 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
 
         int phase = P.two_phase ? 1 : 2;
         bool predicate = false;  // this iteration's S1 seeds Active with the impacted vertices
-        bool bits = true;        // the current frontier is in the bitmap (seeds set bits), else in M
+        bool bits = !InitOf<L>::ALL_ACTIVE;  // the frontier is in the bitmap (seeds set bits), else in M
         bool pull = false;       // this iteration is the NEXT-1 pull over uncertified vertices
         uint32_t iters = 0, n_edges = 0, n_upd = 0, n_read = 0;  // (edge, query) pairs / edge reads
         for (;;) {
@@ -1041,7 +1076,7 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
         transpose_out<L>(P, P.out, q0, nq, xs);
         if (P.stats) {  // reached / precise per query (the thread's query q is fixed)
             const uint32_t q = (uint32_t)(tid % Q);
-            const uint32_t sb = (int)q < nq ? __ldg(P.srcs + q0 + q) : 0xffffffffu;
+            const uint32_t sb = ((int)q < nq && P.srcs) ? __ldg(P.srcs + q0 + q) : 0xffffffffu;
             const uint32_t init = L::decode(L::init_word(), 0);
             unsigned long long r = 0, pr = 0;
             if ((int)q < nq)
@@ -1105,6 +1140,7 @@ void launch_kind_b(int kind, int lw, const BParams& P, int sms, cudaStream_t s) 
         if (lw == 1) launch_b<CG_REACH, PACKED, 1>(P, sms, s);
         else launch_b<CG_REACH, PACKED, 32>(P, sms, s);
         break;
+    case CG_WCC: launch_b<CG_WCC, PACKED, 2>(P, sms, s); break;
     default: throw Error(CG_EINVAL, "bad kind");
     }
 }
@@ -1114,6 +1150,7 @@ void launch_kind_b(int kind, int lw, const BParams& P, int sms, cudaStream_t s) 
 // for Viterbi (CG_LANES=32 forces u32 lanes for every kind).
 int lane_width(const Graph& G, int kind) {
     const char* e = getenv("CG_LANES");
+    if (kind == CG_WCC) return 2;  // labels
     if (e && atoi(e) == 32) return 32;
     if (kind == CG_REACH) return 1;
     if (kind == CG_VITERBI) return (e && atoi(e) == 33) ? 33 : 32;  // CG_LANES=33: 32 per pass (measured slower)
@@ -1138,7 +1175,7 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
         w.n = G.n;
         w.B = 16;
     }
-    const int Q = lw == 32 ? 16 : 32;  // (lw 33: u32 lanes, 32 per pass)
+    const int Q = lw == 2 ? 1 : lw == 32 ? 16 : 32;  // (lw 33: u32 lanes, 32 per pass; lw 2: WCC labels)
     DevBuf<unsigned long long> st;
     if (stats) st.alloc((size_t)c.n_src * NSTAT, s);
     BParams P{};
@@ -1243,7 +1280,7 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
             o.scanned_p1 = (int64_t)x[ST_S1];
             o.scanned_p2 = (int64_t)x[ST_S2];
             o.batch_queries = Q;
-            o.row_bytes = lw == 1 ? 4 : lw == 33 ? 128 : 64;
+            o.row_bytes = (lw == 1 || lw == 2) ? 4 : lw == 33 ? 128 : 64;
         }
     }
 }

@@ -43,6 +43,8 @@ struct Core {
     // queries' values kept as rows hub_vals[v][0..2K) = (Q(h_k) on G at v | Q(h_k) on G^R at v)
     DevBuf<uint32_t> hub_vals;
     uint32_t hub_k = 0;
+    Adj sym;               // WCC: CG ∪ CG^R (built on the first WCC 2Phase query)
+    bool sym_built = false;
 };
 
 struct Workspace {
@@ -87,12 +89,14 @@ struct Graph {
     Adj g;                 // CSR of G
     Adj gr;                // CSR of G^R (= CSC of G)
     DevBuf<uint32_t> reid; // CSC position -> CSR edge index
-    Core core[6];          // indexed by cg_kind (BFS uses the REACH slot: one general CG)
+    Core core[6];          // indexed by cg_kind (BFS and WCC use the REACH slot: one general CG)
+    Adj gsym;              // WCC: G ∪ G^R (built on the first WCC query)
+    bool gsym_built = false;
     Workspace ws;
     BatchSpace bs;
 };
 
-inline int core_slot(int kind) { return kind == CG_BFS ? CG_REACH : kind; }
+inline int core_slot(int kind) { return (kind == CG_BFS || kind == CG_WCC) ? CG_REACH : kind; }
 
 // graph_build.cu
 void build_graph(Graph& G, int64_t n, int64_t m, const uint32_t* src, const uint32_t* dst, const uint32_t* w,
@@ -123,6 +127,7 @@ void build_core_partial(Graph& G, int kind, int32_t K, int policy, const uint32_
 void build_core_from_flags(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs, uint64_t seed,
                            const uint8_t* flags, int connectivity, cudaStream_t s);
 void save_core(Graph& G, int kind, const char* path, cudaStream_t s);
+void ensure_wcc_graphs(Graph& G, bool two_phase, cudaStream_t s);  // G ∪ G^R, CG ∪ CG^R for WCC
 void load_core(Graph& G, int kind, const char* path, cudaStream_t s);
 void build_core(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs, uint64_t seed, int alg,
                 int connectivity, cudaStream_t s);

@@ -11,7 +11,7 @@ import torch
 
 from . import _lib
 
-KINDS = {"sssp": 0, "sswp": 1, "ssnp": 2, "viterbi": 3, "bfs": 4, "reach": 5}
+KINDS = {"sssp": 0, "sswp": 1, "ssnp": 2, "viterbi": 3, "bfs": 4, "reach": 5, "wcc": 6}
 MODES = {"2phase": 0, "full": 1}
 HUB_POLICIES = {"topdeg": 0, "sampled": 1, "given": 2}
 CG_ALGS = {"auto": 0, "specialized": 1, "general": 2, "general_perdir": 3}
@@ -209,6 +209,8 @@ class Graph:
         p1=True (or a uint32 [n_src, n] tensor) also returns the phase-1 values (2phase only).
         stats=True returns per-query counters (synchronises)."""
         k = kind_id(kind)
+        if k == KINDS["wcc"] and sources is None:  # whole-graph query: one row of labels
+            sources = [0]
         src = _u32(sources, self.device).reshape(-1)
         ns = src.numel()
         if out is None:

@@ -411,3 +411,43 @@ def test_core_graph_save_load(tmp_path):
         g3.load_core("sssp", str(tmp_path / "sssp.cg"))
     with pytest.raises(CGInvalid):
         g3.load_core("sssp", str(tmp_path / "missing.cg"))
+
+
+@pytest.mark.parametrize("seed", range(3))
+def test_wcc_small_random(seed):
+    """NEXT-3 WCC: labels (minimum id of the weak component) from FULL and 2PHASE equal the
+    oracle on random multigraphs (isolated vertices, duplicates, self-loops); phase-1 labels
+    equal the oracle's WCC of the Core Graph alone (label propagation on CG ∪ CG^R from the
+    vertex ids converges to the CG's weak components: reading W2)."""
+    rng = np.random.default_rng(100 + seed)
+    n = int(rng.integers(2, 400))
+    src, dst, w = random_multigraph(rng, n, int(rng.integers(0, 3 * n + 1)))
+    g, og = both(n, src, dst, w)
+    ogr = oracle.transpose(og)
+    exp = oracle.wcc(og)
+    g.build("wcc", K=min(8, n))
+    flags = oracle.cg_alg2(og, ogr, oracle.hubs_topdeg(og, ogr, min(8, n)), per_direction=True)
+    assert np.array_equal(g.core_flags("wcc").cpu().numpy(), flags)
+    for mode in ("full", "2phase"):
+        out = to_np(g.query("wcc", None, mode=mode))
+        assert out.shape == (1, n)
+        assert np.array_equal(out[0], exp), mode
+    _, p1 = g.query("wcc", None, mode="2phase", p1=True)
+    assert np.array_equal(to_np(p1)[0], oracle.wcc(oracle.subgraph(og, flags)))
+
+
+def test_wcc_rmat_and_errors():
+    from paper_conf_eurosys_0002a0a024_b200 import CGInvalid
+    n, m = 1 << 15, 8 << 15
+    src, dst, w = gen.rmat(n, m, seed=71)
+    g, og = both(n, src, dst, w)
+    exp = oracle.wcc(og)
+    g.build("reach", K=20)  # WCC shares REACH's general CG
+    for mode in ("full", "2phase"):
+        out, st = g.query("wcc", None, mode=mode, stats=True)
+        assert np.array_equal(to_np(out)[0], exp), mode
+        assert st[0]["batch_queries"] == 1
+    with pytest.raises(CGInvalid):
+        g.query("wcc", to_dev(np.array([0, 1], np.uint32)), mode="full")
+    host = g.query_host("wcc", np.array([0], np.uint32), mode="2phase")
+    assert np.array_equal(host.numpy()[0], exp)

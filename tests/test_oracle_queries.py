@@ -13,6 +13,7 @@ import pytest
 import scipy.sparse as sp
 from scipy.sparse.csgraph import breadth_first_order, dijkstra
 
+import gen
 import oracle
 from helpers import INF32, KINDS, brute_force, np_canonical, random_multigraph, rmat_small
 
@@ -178,3 +179,29 @@ def test_init_values_reading_q1():
     f = lambda x: int(np.array([x], dtype=np.float32).view(np.uint32)[0])
     assert [oracle.init_val(k) for k in KINDS] == [INF32, 0, INF32, f(0.0), INF32, 0]
     assert [oracle.source_val(k) for k in KINDS] == [0, INF32, 0, f(1.0), 0, 1]
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_wcc_oracle_pins(seed):
+    """NEXT-3 WCC (Table 6 WCC row): the label fixpoint is the minimum vertex id of
+    the weak component.  Pinned against scipy's weak connected components (an independent
+    algorithm) plus the invariants label(v) <= v, label(label(v)) == label(v), and equal labels
+    at both ends of every edge."""
+    import scipy.sparse as sp
+    import scipy.sparse.csgraph as csg
+    rng = np.random.default_rng(seed)
+    n = int(rng.integers(1, 3000))
+    src, dst, w = gen.rmat(max(n, 2), int(rng.integers(0, 3 * n + 1)), seed=seed + 11) if n > 1 else (
+        np.zeros(0, np.uint32), np.zeros(0, np.uint32), np.zeros(0, np.uint32))
+    n = max(n, 2)
+    g = oracle.canonical_csr(n, src, dst, w)
+    lab = oracle.wcc(g)
+    a = sp.csr_matrix((np.ones(g.m), g.col, g.ptr), shape=(n, n))
+    nc, comp = csg.connected_components(a, directed=True, connection="weak")
+    mins = np.full(nc, n)
+    np.minimum.at(mins, comp, np.arange(n))
+    assert np.array_equal(lab, mins[comp].astype(np.uint32))
+    assert np.all(lab <= np.arange(n)) and np.array_equal(lab[lab], lab)
+    rows = np.repeat(np.arange(n), np.diff(g.ptr))
+    assert np.array_equal(lab[rows], lab[g.col])
+    assert np.array_equal(oracle.query("wcc", g, 0), lab)
