@@ -1,6 +1,13 @@
 #!/usr/bin/env python
-"""CG quality on a config: edge fraction, phase-1 precision, 2Phase vs FULL edges, for chosen CG
-algorithms / hub policies (Table 4 / Table 5 analogs, SURVEY config 5 sweep)."""
+"""CG quality on a config: edge fraction, phase-1 precision, 2Phase vs FULL edges and time, for
+chosen CG algorithms / hub policies / hub counts — the Table 4 (CG %E), Table 5 (precision) and
+Fig 3 / Table 13 (K) analogs; BASELINE.json configs[4] is the K sweep on C5:
+
+    python tools/cg_quality.py --config c5 --kinds sssp,sswp,reach --K 5,10,20,40,60,80,100 \
+        --policy topdeg,sampled --sources 10 > profiles/r1_ksweep_c5.jsonl
+
+End-to-end speedup = FULL ms / 2Phase ms for the same batch of sources (one cg_query call each,
+CUDA events, median of --reps after one warm-up); build_ms is the Core Graph build (a3-a7)."""
 import argparse
 import json
 import os
@@ -18,6 +25,7 @@ def main():
     p.add_argument("--K", default="20")
     p.add_argument("--policy", default="topdeg")
     p.add_argument("--sources", type=int, default=16)
+    p.add_argument("--reps", type=int, default=3)
     a = p.parse_args()
     import numpy as np
     import torch
@@ -45,12 +53,28 @@ def main():
                     prec = sum(x["precise_p1"] for x in st)
                     e2 = sum(x["edges_p1"] + x["edges_p2"] for x in st)
                     ef = sum(x["edges_p2"] for x in stf)
+
+                    def timed(mode):
+                        g.query(kind, srcs, mode=mode)
+                        ts = []
+                        for _ in range(a.reps):
+                            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                            torch.cuda.synchronize()
+                            e0.record()
+                            g.query(kind, srcs, mode=mode)
+                            e1.record()
+                            torch.cuda.synchronize()
+                            ts.append(e0.elapsed_time(e1))
+                        return sorted(ts)[len(ts) // 2]
+                    ms2, msf = timed("2phase"), timed("full")
                     per_q = [round(100 * x["precise_p1"] / x["reached"], 2) if x["reached"] else 100.0 for x in st]
                     print(json.dumps({"config": cfg.name, "kind": kind, "alg": alg, "K": K, "policy": policy,
                                       "cg_edge_pct": round(100 * info["edge_fraction"], 3),
                                       "p1_precision_pct": round(100 * prec / max(reached, 1), 3),
                                       "min_query_precision_pct": min(per_q), "edges_2phase_over_full": round(e2 / max(ef, 1), 3),
-                                      "build_ms": round(info["build_ms"], 1)}), flush=True)
+                                      "build_ms": round(info["build_ms"], 1), "n_sources": len(srcs),
+                                      "ms_2phase": round(ms2, 3), "ms_full": round(msf, 3),
+                                      "speedup_2phase_vs_full": round(msf / ms2, 3)}), flush=True)
 
 
 if __name__ == "__main__":
