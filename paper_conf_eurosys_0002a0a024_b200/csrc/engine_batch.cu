@@ -20,6 +20,7 @@
 #include <cstdlib>
 
 #include <cuda_fp16.h>
+#include <type_traits>
 
 #include "kernels.cuh"
 
@@ -89,11 +90,22 @@ struct Lanes32 {  // one u32 per query (Table 6 types), QN queries per pass
     __device__ static void seed(uint32_t* p, uint32_t, uint32_t val) { *p = val; }
     __device__ static uint32_t src_val() { return O::SRC; }
     __device__ static uint32_t nb_val(uint32_t w) { return O::ext(O::SRC, w); }
-    __device__ static uint32_t relax(uint32_t* p, const uint32_t (&u)[G], const uint32_t (&c)[G], uint32_t w,
+    static constexpr bool VIT = KIND == CG_VITERBI;
+    using Arg = typename std::conditional<VIT, VitArg, uint32_t>::type;  // per-edge, shared by the row
+    __device__ static Arg arg(uint32_t w) {
+        if constexpr (VIT) return vit_arg(w);
+        else return w;
+    }
+    __device__ static uint32_t relax(uint32_t* p, const uint32_t (&u)[G], const uint32_t (&c)[G], const Arg& w,
                                      uint32_t act, uint32_t& n_edges, uint32_t& n_upd, uint32_t*) {
         if (!act || u[0] == O::INIT) return 0u;  // (a pull may read an unreached u)
         ++n_edges;
-        const uint32_t cand = O::ext(u[0], w);
+        uint32_t cand;
+        if constexpr (VIT) {
+            cand = vit_div(u[0], w);
+        } else {
+            cand = O::ext(u[0], w);
+        }
         if (!O::better(cand, c[0])) return 0u;  // Needed(e(u,v))
         O::edge_fn(p, cand);                  // EdgeFunction
         ++n_upd;
@@ -113,6 +125,8 @@ template <int KIND>
 struct Lanes16 {
     static_assert(KIND == CG_SSSP || KIND == CG_SSWP || KIND == CG_SSNP || KIND == CG_BFS, "f16 lanes");
     static constexpr int Q = 32, QPW = 2, RW = 16, G = 4;
+    using Arg = uint32_t;
+    __device__ static Arg arg(uint32_t w) { return w; }
     static constexpr bool MAXK = KIND == CG_SSWP;
     static constexpr uint32_t INF16 = 0x7c00u, LIMIT = 0x68006800u;  // +inf; 2048.0 in both lanes
     static constexpr uint32_t INIT16 = MAXK ? 0u : INF16, SRC16 = MAXK ? INF16 : 0u;
@@ -139,31 +153,45 @@ struct Lanes16 {
         else r = __hadd2(a, b);  // SSSP: + w; BFS: + 1
         return *reinterpret_cast<const uint32_t*>(&r);
     }
-    // Process + EdgeFunction of one 16 B chunk (4 words, 8 queries); act: 8 query bits
-    __device__ static uint32_t relax(uint32_t* p, const uint32_t (&u)[G], const uint32_t (&c)[G], uint32_t w,
+    __device__ static uint32_t needed2(uint32_t x, uint32_t c) {  // 0xffff per lane whose candidate is better
+        const __half2 a = *reinterpret_cast<const __half2*>(&x), b = *reinterpret_cast<const __half2*>(&c);
+        return MAXK ? __hgt2_mask(a, b) : __hlt2_mask(a, b);
+    }
+    // Process + EdgeFunction of one 16 B chunk (4 words, 8 queries); act: 8 query bits.
+    // The Needed test is taken on every lane, not only the active ones: a lane whose u is not
+    // active for its query holds a value already pushed along (u, v), so its candidate is never
+    // better than Val(v) — except against a stale pre-read, where applying it is still a valid
+    // relaxation (a real path value) and v becomes active for that query (reading N1).  The
+    // EdgeFunction therefore sends the candidates themselves: a non-needed lane's candidate is no
+    // better than the current Val(v) and leaves it unchanged.  Common case (nothing needed): one
+    // packed ⊕, one packed compare and an OR per word.
+    __device__ static uint32_t relax(uint32_t* p, const uint32_t (&u)[G], const uint32_t (&c)[G], Arg w,
                                      uint32_t act, uint32_t& n_edges, uint32_t& n_upd, uint32_t* err) {
         if (!act) return 0u;
         n_edges += __popc(act);
         const uint32_t w2 = (KIND == CG_BFS ? 0x3c00u : h16(w)) * 0x10001u;
-        uint32_t cand[G], ch = 0, over = 0;
+        uint32_t x[G], bm[G], any = 0;
 #pragma unroll
         for (int i = 0; i < G; ++i) {
-            const uint32_t am = halves2(act >> (2 * i));
-            const uint32_t x = ext2(u[i], w2);
-            const uint32_t bm = (MAXK ? __vcmpgtu2(x, c[i]) : __vcmpltu2(x, c[i])) & am;  // Needed, 2 queries
-            if (KIND == CG_SSSP || KIND == CG_BFS) over |= __vcmpgeu2(x, LIMIT) & bm;
-            cand[i] = MAXK ? (x & bm) : ((x & bm) | (INF16 * 0x10001u & ~bm));  // others neutral
-            ch |= bits2(bm) << (2 * i);
+            x[i] = ext2(u[i], w2);
+            bm[i] = needed2(x[i], c[i]);
+            any |= bm[i];
+        }
+        if (!any) return 0u;
+        uint32_t ch = 0, over = 0;
+#pragma unroll
+        for (int i = 0; i < G; ++i) {
+            if (KIND == CG_SSSP || KIND == CG_BFS) over |= __vcmpgeu2(x[i], LIMIT) & bm[i];
+            ch |= bits2(bm[i]) << (2 * i);
         }
         if (over) atomicOr(err, ERR_LANE_OVERFLOW);
-        if (!ch) return 0u;
         if (MAXK)
-            asm volatile("red.relaxed.gpu.global.max.noftz.v4.f16x2 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(cand[0]),
-                         "r"(cand[1]), "r"(cand[2]), "r"(cand[3])
+            asm volatile("red.relaxed.gpu.global.max.noftz.v4.f16x2 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(x[0]),
+                         "r"(x[1]), "r"(x[2]), "r"(x[3])
                          : "memory");
         else
-            asm volatile("red.relaxed.gpu.global.min.noftz.v4.f16x2 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(cand[0]),
-                         "r"(cand[1]), "r"(cand[2]), "r"(cand[3])
+            asm volatile("red.relaxed.gpu.global.min.noftz.v4.f16x2 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(x[0]),
+                         "r"(x[1]), "r"(x[2]), "r"(x[3])
                          : "memory");
         n_upd += __popc(ch);
         return ch;
@@ -173,6 +201,8 @@ struct Lanes16 {
 // one bit per query (REACH): InitVal 0, SourceInitVal 1, cand = u; EdgeFunction red.or
 struct LanesBit {
     static constexpr int Q = 32, QPW = 32, RW = 1, G = 1;
+    using Arg = uint32_t;
+    __device__ static Arg arg(uint32_t w) { return w; }
     __device__ static uint32_t init_word() { return 0u; }
     __device__ static uint32_t decode(uint32_t x, uint32_t j) { return (x >> j) & 1u; }
     __device__ static uint32_t live(uint32_t x) { return x; }
@@ -195,6 +225,8 @@ struct LanesBit {
 // active at the start of both phases (reading W2), cand = Val(u), select min (red.min).
 struct LanesLabel {
     static constexpr int Q = 1, QPW = 1, RW = 1, G = 1;
+    using Arg = uint32_t;
+    __device__ static Arg arg(uint32_t w) { return w; }
     static constexpr bool ALL_ACTIVE = true;
     __device__ static uint32_t init_word() { return 0xffffffffu; }  // (never a label: the stats' "unreached")
     __device__ static uint32_t init_at(uint64_t i) { return (uint32_t)i; }
@@ -428,10 +460,8 @@ __device__ void compact_bits(const BParams& P, const GraphView& g, unsigned long
 }
 
 // S1 for large frontiers held as query masks M (F_MASKS, and F_IMPACTED / F_UNCERT after their
-// mark pass): no bitmap.  A warp takes 32 bitmap-word spans (1024 vertices) and issues the masks
-// and row offsets of 16 words (512 vertices) at once — one memory round trip per half instead of
-// a dependent degree fetch per active word.  Pass 1 counts and reserves the CTA's list range;
-// pass 2 re-reads (L2), writes the list and consumes the masks (deg-0 vertices included).
+// mark pass): no bitmap.  A warp issues the masks and row offsets of 16 bitmap words (512
+// vertices) at once — one memory round trip instead of a dependent degree fetch per active word.
 __device__ __forceinline__ void span_loads(const BParams& P, const GraphView& g, uint32_t g0, uint32_t w1, int h,
                                            uint32_t (&mv)[16], uint32_t (&dg)[16]) {
     const uint32_t lane = threadIdx.x & 31;
@@ -456,79 +486,78 @@ __device__ __forceinline__ void span_loads(const BParams& P, const GraphView& g,
 
 __device__ void compact_masks(const BParams& P, const GraphView& g, unsigned long long* cnt_slot,
                               unsigned long long* act_slot, uint32_t* sm) {
+    // One pass: the CTA's word range is taken in rounds of BW half-spans (16 words = 512
+    // vertices per warp); a round's masks and degrees stay in registers while the CTA reserves
+    // its list range (one 64-bit atomicAdd per round), then the entries are written and the
+    // masks consumed.  List order is vertex order within a round; S2 needs only that the edge
+    // offsets ascend with the list index, which the packed (count, edges) reservation gives.
     const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const uint64_t W = P.words;
     const uint32_t w0 = (uint32_t)(W * blockIdx.x / gridDim.x), w1 = (uint32_t)(W * (blockIdx.x + 1) / gridDim.x);
     const uint32_t lt = (1u << lane) - 1u;
-    uint32_t cnt = 0, edges = 0, active = 0;
-    for (uint32_t g0 = w0 + warp * 32; g0 < w1; g0 += BW * 32)
+    uint32_t active = 0;
+    for (uint32_t r0 = w0; r0 < w1; r0 += BW * 16) {
+        const uint32_t g0 = r0 + warp * 16;
+        uint32_t mv[16], dg[16];
+        span_loads(P, g, g0, w1, 0, mv, dg);
+        uint32_t cnt = 0, edges = 0;
 #pragma unroll
-        for (int h = 0; h < 2; ++h) {
-            uint32_t mv[16], dg[16];
-            span_loads(P, g, g0, w1, h, mv, dg);
-#pragma unroll
-            for (int j = 0; j < 16; ++j) {
-                active += mv[j] != 0u;
-                cnt += dg[j] != 0u;
-                edges += dg[j];
+        for (int j = 0; j < 16; ++j) {
+            active += mv[j] != 0u;
+            cnt += dg[j] != 0u;
+            edges += dg[j];
+        }
+        for (int o = 16; o > 0; o >>= 1) {
+            cnt += __shfl_xor_sync(FULL, cnt, o);
+            edges += __shfl_xor_sync(FULL, edges, o);
+        }
+        if (lane == 0) {
+            sm[warp] = cnt;
+            sm[BW + warp] = edges;
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            uint32_t tc = 0, te = 0;
+            for (int i = 0; i < BW; ++i) {
+                const uint32_t c = sm[i], e = sm[BW + i];
+                sm[i] = tc;
+                sm[BW + i] = te;
+                tc += c;
+                te += e;
             }
+            unsigned long long old = 0;
+            if (tc) old = atomicAdd(cnt_slot, ((unsigned long long)tc << 32) | te);
+            sm[2 * BW] = (uint32_t)(old >> 32);
+            sm[2 * BW + 1] = (uint32_t)old;
         }
-    for (int o = 16; o > 0; o >>= 1) {
-        cnt += __shfl_xor_sync(FULL, cnt, o);
-        edges += __shfl_xor_sync(FULL, edges, o);
-        active += __shfl_xor_sync(FULL, active, o);
-    }
-    if (lane == 0) {
-        sm[warp] = cnt;
-        sm[BW + warp] = edges;
-        if (active) atomicAdd(act_slot, (unsigned long long)active);
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        uint32_t tc = 0, te = 0;
-        for (int i = 0; i < BW; ++i) {
-            const uint32_t c = sm[i], e = sm[BW + i];
-            sm[i] = tc;
-            sm[BW + i] = te;
-            tc += c;
-            te += e;
-        }
-        unsigned long long old = 0;
-        if (tc) old = atomicAdd(cnt_slot, ((unsigned long long)tc << 32) | te);
-        sm[2 * BW] = (uint32_t)(old >> 32);
-        sm[2 * BW + 1] = (uint32_t)old;
-    }
-    __syncthreads();
-    uint32_t pos = sm[2 * BW] + sm[warp];
-    uint32_t eb = sm[2 * BW + 1] + sm[BW + warp];
-    __syncthreads();
-    for (uint32_t g0 = w0 + warp * 32; g0 < w1; g0 += BW * 32)
+        __syncthreads();
+        uint32_t pos = sm[2 * BW] + sm[warp];
+        uint32_t eb = sm[2 * BW + 1] + sm[BW + warp];
+        __syncthreads();  // sm is rewritten by the next round
 #pragma unroll
-        for (int h = 0; h < 2; ++h) {
-            uint32_t mv[16], dg[16];
-            span_loads(P, g, g0, w1, h, mv, dg);
+        for (int j = 0; j < 16; ++j) {
+            const uint32_t v = (g0 + j) * 32 + lane;
+            if (mv[j]) P.M[v] = 0u;  // consumed
+            const uint32_t d = dg[j];
+            uint32_t incl = d;
 #pragma unroll
-            for (int j = 0; j < 16; ++j) {
-                const uint32_t v = (g0 + h * 16 + j) * 32 + lane;
-                if (mv[j]) P.M[v] = 0u;  // consumed
-                const uint32_t d = dg[j];
-                uint32_t incl = d;
-#pragma unroll
-                for (int o = 1; o < 32; o <<= 1) {
-                    const uint32_t y = __shfl_up_sync(FULL, incl, o);
-                    if (lane >= (uint32_t)o) incl += y;
-                }
-                const uint32_t bal = __ballot_sync(FULL, d != 0);
-                if (d) {
-                    const uint32_t i = pos + __popc(bal & lt);
-                    P.lv[i] = v;
-                    P.lo[i] = eb + incl - d;
-                    P.lm[i] = mv[j];
-                }
-                pos += __popc(bal);
-                eb += __shfl_sync(FULL, incl, 31);
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t y = __shfl_up_sync(FULL, incl, o);
+                if (lane >= (uint32_t)o) incl += y;
             }
+            const uint32_t bal = __ballot_sync(FULL, d != 0);
+            if (d) {
+                const uint32_t i = pos + __popc(bal & lt);
+                P.lv[i] = v;
+                P.lo[i] = eb + incl - d;
+                P.lm[i] = mv[j];
+            }
+            pos += __popc(bal);
+            eb += __shfl_sync(FULL, incl, 31);
         }
+    }
+    for (int o = 16; o > 0; o >>= 1) active += __shfl_xor_sync(FULL, active, o);
+    if (lane == 0 && active) atomicAdd(act_slot, (unsigned long long)active);
 }
 
 // Mark passes (thread per vertex, coalesced): F_IMPACTED — Alg 3 l.15, M[v] = the queries for
@@ -640,7 +669,8 @@ __device__ __forceinline__ void window_edges(const BParams& P, const GraphView& 
             const uint32_t mk = __shfl_sync(FULL, mask, kk & 31u);
             if (kk == NONE) continue;
             ++n_read;
-            const uint32_t d = sd[s], w = sw[s];
+            const uint32_t d = sd[s];
+            const typename L::Arg w = L::arg(sw[s]);         // per edge, shared by the row's queries
             const uint32_t* rv = vs + (s * 32 + lane) * RW;  // v's row (swizzled copies)
             const uint32_t* ru = xs + kk * RW;               // u's row
             uint32_t* pv = P.V + (size_t)d * RW;
@@ -820,8 +850,9 @@ __device__ void relax_pull(const BParams& P, uint32_t count, uint32_t E, uint32_
 #pragma unroll
             for (int u = 0; u < U; ++u) {
                 if (!ok[u]) continue;
-                uint32_t src, w;
-                wd[u].decode(P.dbits, P.dmask, src, w);
+                uint32_t src, w0;
+                wd[u].decode(P.dbits, P.dmask, src, w0);
+                const typename L::Arg w = L::arg(w0);
                 ++n_read;
                 const uint32_t* ru = P.V + (size_t)src * RW;  // u's row (L1: a stale value is never better)
                 uint32_t* pv = P.V + (size_t)vk[u] * RW;

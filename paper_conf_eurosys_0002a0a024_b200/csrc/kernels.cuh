@@ -40,6 +40,28 @@ template <> struct Op<CG_VITERBI> {
     __device__ static bool better(uint32_t a, uint32_t b) { return a > b; }
     __device__ static void edge_fn(uint32_t* p, uint32_t v) { red_max(p, v); }
 };
+// Viterbi's Val(u)/w rounded to nearest (reading Q13), with the per-edge reciprocal hoisted out
+// of a batch row: for w <= 64 and x = Val(u) >= 2^-64, r = RN(1/w) once per edge, q = RN(x*r),
+// the residual e = x - q*w exactly (one FMA), and Markstein's correction RN(q + e*r) — equal
+// to RN(x/w) for every such x and w.  tests/test_viterbi_div.py checks that exhaustively (all
+// 2^23 significands of three binades x every w <= 64); within the fast range neither the
+// quotient nor the residual leaves the normal range, so each result scales exactly with x's
+// exponent and the three binades cover it.  Otherwise: __fdiv_rn.
+struct VitArg {
+    uint32_t w;
+    float r;  // RN(1/w), or 0 (slow path)
+};
+__device__ __forceinline__ VitArg vit_arg(uint32_t w) { return {w, w <= 64u ? __frcp_rn((float)w) : 0.0f}; }
+__device__ __forceinline__ uint32_t vit_div(uint32_t a, const VitArg& A) {
+    const float x = __uint_as_float(a);
+    const float b = __uint2float_rn(A.w);  // exact for w <= 64
+    const float q = __fmul_rn(x, A.r);
+    const float e = __fmaf_rn(-q, b, x);
+    float y = __fmaf_rn(e, A.r, q);
+    if (!(A.r != 0.0f && x >= 0x1p-64f)) y = __fdiv_rn(x, b);  // rare: large w or a tiny value
+    return __float_as_uint(y);
+}
+
 template <> struct Op<CG_BFS> {
     static constexpr uint32_t INIT = 0xffffffffu, SRC = 0u;
     __device__ static uint32_t ext(uint32_t a, uint32_t) { return a + 1u; }
