@@ -36,6 +36,10 @@ constexpr int BW = BT / 32;      // warps per CTA
 #define CGB_STAGES 2
 #endif
 constexpr int S_PIPE = CGB_STAGES;  // value-row pipeline depth (chunks of 32 edges per warp)
+#ifndef CGB_EAHEAD
+#define CGB_EAHEAD CGB_STAGES
+#endif
+constexpr int E_AHEAD = CGB_EAHEAD;  // edge-word lead over the row requests (chunks)
 
 enum { ST_IT1, ST_IT2, ST_E1, ST_E2, ST_U1, ST_U2, ST_F1, ST_F2, ST_IMP, ST_REACH, ST_PREC, ST_S1, ST_S2, NSTAT };
 enum { CT0 = 8, CTS = 2, CT_LIST = 0, CT_ACTIVE = 1 };
@@ -597,15 +601,17 @@ template <class L> struct RowCopy {
 // The edges [e, ehi) of one 32-row window: lane r of the window holds row r's first edge index
 // `off`, its address base (edge address = base + edge index) and its query mask; the rows'
 // values are in xs (r * RW + word).  Lane L takes edge L of each 32-edge chunk for all Q queries.
-// Software pipeline (S_PIPE stages, per-warp ring `vs` in shared memory): the edge word of chunk
-// c + S is loaded when chunk c + S - 1's value rows are requested (cp.async global -> shared),
-// while chunk c is consumed.
+// Software pipeline (per-warp ring `vs` of S_PIPE value-row stages in shared memory; E_AHEAD
+// edge-word slots in registers): while chunk c is consumed, chunk c + S - 1's value rows are
+// requested (cp.async global -> shared) and the edge words of chunk c + S - 1 + E_AHEAD are
+// loaded — the edge stream runs E_AHEAD chunks ahead of the row gathers it feeds.
 template <int KIND, bool PACKED, class L>
 __device__ __forceinline__ void window_edges(const BParams& P, const GraphView& g, const uint32_t* xs, uint32_t* vs,
                                              uint32_t off, uint32_t base, uint32_t mask, uint32_t e, uint32_t ehi,
                                              bool set_bits, bool fresh, uint32_t& n_edges, uint32_t& n_upd,
                                              uint32_t& n_read) {
-    constexpr int S = S_PIPE, RW = L::RW;
+    constexpr int S = S_PIPE, EA = E_AHEAD, RW = L::RW;
+    static_assert(EA % S == 0 && EA >= S, "E_AHEAD must be a multiple of S_PIPE");
     using RC = RowCopy<L>;
     constexpr uint32_t NONE = 0xffffffffu;
     const uint32_t lane = threadIdx.x & 31;
@@ -613,9 +619,9 @@ __device__ __forceinline__ void window_edges(const BParams& P, const GraphView& 
     if (e >= ehi) return;
     const uint32_t nch = (ehi - e + 31) >> 5;
 
-    EdgeWord<PACKED> ew[S];        // fetched edge words, chunk c + S ahead
-    uint32_t ek[S];                // their window row (NONE: no edge / inactive row)
-    uint32_t sd[S], sw[S], sk[S];  // requested chunks: destination, weight, window row
+    EdgeWord<PACKED> ew[EA];       // fetched edge words (slot = chunk % EA)
+    uint32_t ek[EA];               // their window row (NONE: no edge / inactive row)
+    uint32_t sd[S], sw[S], sk[S];  // requested chunks (slot = chunk % S): destination, weight, window row
 
     auto fetch = [&](uint32_t c, EdgeWord<PACKED>& wd, uint32_t& kout) {
         const uint32_t t = e + c * 32 + lane;
@@ -629,23 +635,39 @@ __device__ __forceinline__ void window_edges(const BParams& P, const GraphView& 
         if (ok) wd.load(g, a);
         kout = ok ? kk : NONE;
     };
+    // Rows of C > 1 copies are gathered cooperatively: copy instruction i moves piece (lane % C)
+    // of the row of lane i * (32 / C) + lane / C, so one instruction touches 32 / C rows of
+    // contiguous 16 B pieces instead of 32 scattered lines (C times fewer L1 tag lookups per
+    // chunk).  The slot is shared across lanes, so the caller brackets it with __syncwarp().
     auto request = [&](int slot, const EdgeWord<PACKED>& wd, uint32_t kk) {
         sk[slot] = kk;
+        uint32_t dd = NONE;
         if (kk != NONE) {
             uint32_t d, w;
             wd.decode(P.dbits, P.dmask, d, w);
             sd[slot] = d;
             sw[slot] = w;
-            const uint32_t* src = P.V + (size_t)d * RW;
-            uint32_t* dst = vs + (slot * 32 + lane) * RW;
+            dd = d;
+        }
+        if constexpr (RC::C > 1) {
+            constexpr uint32_t RPI = 32 / RC::C;  // rows per copy instruction
+            const uint32_t p = lane % RC::C;
 #pragma unroll
-            for (uint32_t i = 0; i < RC::C; ++i) RC::copy(dst + RC::CW4 * (i ^ swz), src + RC::CW4 * i, fresh);
+            for (uint32_t i = 0; i < RC::C; ++i) {
+                const uint32_t r = i * RPI + lane / RC::C;
+                const uint32_t dr = __shfl_sync(FULL, dd, r);
+                if (dr != NONE)
+                    RC::copy(vs + (slot * 32 + r) * RW + RC::CW4 * (p ^ RC::sw(r)), P.V + (size_t)dr * RW + RC::CW4 * p,
+                             fresh);
+            }
+        } else if (dd != NONE) {
+            RC::copy(vs + (slot * 32 + lane) * RW, P.V + (size_t)dd * RW, fresh);
         }
         cp_async_commit();
     };
 
 #pragma unroll
-    for (int s = 0; s < S; ++s) {
+    for (int s = 0; s < EA; ++s) {
         ek[s] = NONE;
         if ((uint32_t)s < nch) fetch(s, ew[s], ek[s]);
     }
@@ -653,25 +675,29 @@ __device__ __forceinline__ void window_edges(const BParams& P, const GraphView& 
     for (int s = 0; s < S - 1; ++s) {
         request(s, ew[s], ek[s]);
         ek[s] = NONE;
-        if ((uint32_t)(s + S) < nch) fetch(s + S, ew[s], ek[s]);
+        if ((uint32_t)(s + EA) < nch) fetch(s + EA, ew[s], ek[s]);
     }
-    for (uint32_t c0 = 0; c0 < nch; c0 += S) {
+    for (uint32_t c0 = 0; c0 < nch; c0 += EA) {
 #pragma unroll
-        for (int s = 0; s < S; ++s) {
+        for (int s = 0; s < EA; ++s) {
             const uint32_t cc = c0 + s;
             if (cc >= nch) break;
-            const int js = (s + S - 1) % S;  // slot of chunk cc + S - 1
-            request(js, ew[js], ek[js]);
-            ek[js] = NONE;
-            if (cc + 2 * S - 1 < nch) fetch(cc + 2 * S - 1, ew[js], ek[js]);
-            cp_async_wait<S - 1>();  // chunk cc's row has landed (this lane's own copies)
-            const uint32_t kk = sk[s];
+            const int je = (s + S - 1) % EA;  // edge slot of chunk cc + S - 1
+            const int jr = (s + S - 1) % S;   // its row slot
+            if constexpr (RC::C > 1) __syncwarp();  // every lane is done with slot jr (chunk cc - 1)
+            request(jr, ew[je], ek[je]);
+            ek[je] = NONE;
+            if (cc + S - 1 + EA < nch) fetch(cc + S - 1 + EA, ew[je], ek[je]);
+            cp_async_wait<S - 1>();  // chunk cc's row pieces this lane copied have landed
+            if constexpr (RC::C > 1) __syncwarp();  // ... and those the other lanes copied
+            const int sr = s % S;    // chunk cc's row slot
+            const uint32_t kk = sk[sr];
             const uint32_t mk = __shfl_sync(FULL, mask, kk & 31u);
             if (kk == NONE) continue;
             ++n_read;
-            const uint32_t d = sd[s];
-            const typename L::Arg w = L::arg(sw[s]);         // per edge, shared by the row's queries
-            const uint32_t* rv = vs + (s * 32 + lane) * RW;  // v's row (swizzled copies)
+            const uint32_t d = sd[sr];
+            const typename L::Arg w = L::arg(sw[sr]);         // per edge, shared by the row's queries
+            const uint32_t* rv = vs + (sr * 32 + lane) * RW;  // v's row (swizzled copies)
             const uint32_t* ru = xs + kk * RW;               // u's row
             uint32_t* pv = P.V + (size_t)d * RW;
             uint32_t changed = 0;
@@ -906,44 +932,60 @@ __device__ __forceinline__ uint32_t value_of(const uint32_t* V, uint32_t v, uint
 
 // rows -> dst[(q0+q)*n + v] for q < nq, 32 vertices per warp through shared memory: the 32
 // rows are read with 16 B loads (coalesced), each lane decodes its vertex's Q values, and every
-// query's 32 values leave as one 128 B streaming store
+// query's 32 values leave as one 128 B streaming store.  A warp keeps TU tiles' loads in flight
+// (registers) before it stages them one at a time through its padded shared tile.
 template <class L>
 __device__ void transpose_out(const BParams& P, uint32_t* dst, int q0, int nq, uint32_t* xs) {
     constexpr int RW = L::RW;
+    constexpr bool V4 = RW % 4 == 0;
+    constexpr int NC = V4 ? RW / 4 : RW;  // loads per lane per tile
+    constexpr int TU = NC >= 8 ? 2 : 4;  // <= 16 x 16 B in flight per lane
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t gw = blockIdx.x * BW + (threadIdx.x >> 5);
     const uint32_t NW = gridDim.x * BW;
-    for (uint32_t v0 = gw * 32; v0 < P.n; v0 += NW * 32) {
-        __syncwarp();
-        if constexpr (RW % 4 == 0) {
+    for (uint32_t v0 = gw * 32; v0 < P.n; v0 += NW * 32 * TU) {
+        uint4 x4[V4 ? TU * NC : 1];
+        uint32_t x1[V4 ? 1 : TU * NC];
 #pragma unroll
-            for (int r = 0; r < RW / 4; ++r) {
-                const uint32_t f = r * 32 + lane;  // 16 B chunk f of the 32 rows
-                const uint32_t v = v0 + f / (RW / 4), c = f % (RW / 4);
-                uint4 x = make_uint4(0, 0, 0, 0);
-                if (v < P.n)
-                    asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];"
-                                 : "=r"(x.x), "=r"(x.y), "=r"(x.z), "=r"(x.w)
-                                 : "l"(reinterpret_cast<const uint4*>(P.V + (size_t)v * RW) + c));
-                uint32_t* t = xs + (f / (RW / 4)) * (RW + 1) + 4 * c;
-                t[0] = x.x;
-                t[1] = x.y;
-                t[2] = x.z;
-                t[3] = x.w;
-            }
-        } else {
+        for (int t = 0; t < TU; ++t) {
+            const uint32_t vt = v0 + t * NW * 32;
 #pragma unroll
-            for (int r = 0; r < RW; ++r) {
-                const uint32_t f = r * 32 + lane;
-                const uint32_t v = v0 + f / RW;
-                xs[(f / RW) * (RW + 1) + f % RW] = v < P.n ? ld_cg(P.V + (size_t)v * RW + f % RW) : 0u;
+            for (int r = 0; r < NC; ++r) {
+                const uint32_t f = r * 32 + lane;  // chunk f of the tile's 32 rows
+                const uint32_t v = vt + f / NC, c = f % NC;
+                if constexpr (V4) {
+                    x4[t * NC + r] = v < P.n ? __ldcg(reinterpret_cast<const uint4*>(P.V + (size_t)v * RW) + c)
+                                             : make_uint4(0, 0, 0, 0);
+                } else {
+                    x1[t * NC + r] = v < P.n ? __ldcg(P.V + (size_t)v * RW + c) : 0u;
+                }
             }
         }
-        __syncwarp();
-        const uint32_t v = v0 + lane;
-        if (v < P.n)
-            for (int q = 0; q < nq; ++q)
-                __stcs(dst + (size_t)(q0 + q) * P.n + v, L::decode(xs[lane * (RW + 1) + q / L::QPW], q % L::QPW));
+#pragma unroll
+        for (int t = 0; t < TU; ++t) {
+            const uint32_t vt = v0 + t * NW * 32;
+            if (vt >= P.n) break;
+            __syncwarp();
+#pragma unroll
+            for (int r = 0; r < NC; ++r) {
+                const uint32_t f = r * 32 + lane;
+                if constexpr (V4) {
+                    uint32_t* d = xs + (f / NC) * (RW + 1) + 4 * (f % NC);
+                    const uint4 x = x4[t * NC + r];
+                    d[0] = x.x;
+                    d[1] = x.y;
+                    d[2] = x.z;
+                    d[3] = x.w;
+                } else {
+                    xs[(f / NC) * (RW + 1) + f % NC] = x1[t * NC + r];
+                }
+            }
+            __syncwarp();
+            const uint32_t v = vt + lane;
+            if (v < P.n)
+                for (int q = 0; q < nq; ++q)
+                    __stcs(dst + (size_t)(q0 + q) * P.n + v, L::decode(xs[lane * (RW + 1) + q / L::QPW], q % L::QPW));
+        }
     }
 }
 
