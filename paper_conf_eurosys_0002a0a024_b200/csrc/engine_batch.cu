@@ -84,9 +84,9 @@ struct BParams {
 //   relax(p, uw, cw, w, act, ...)  Process + EdgeFunction of one word (Alg 3 l.22-27): the lanes
 //       of act whose candidate ext(uw, w) is better than cw; returns the changed lanes
 template <int KIND, int QN>
-struct Lanes32 {  // one u32 per query (Table 6 types), QN queries per pass
+struct Lanes32 {  // one u32 per query (Table 6 types), QN queries per pass, 4 words (16 B) per relax group
     using O = Op<KIND>;
-    static constexpr int Q = QN, QPW = 1, RW = QN, G = 1;
+    static constexpr int Q = QN, QPW = 1, RW = QN, G = 4;
     __device__ static uint32_t init_word() { return O::INIT; }
     __device__ static uint32_t decode(uint32_t x, uint32_t) { return x; }
     __device__ static uint32_t live(uint32_t x) { return x != O::INIT; }
@@ -100,20 +100,31 @@ struct Lanes32 {  // one u32 per query (Table 6 types), QN queries per pass
         if constexpr (VIT) return vit_arg(w);
         else return w;
     }
+    // Process + EdgeFunction of 4 queries: candidates and Needed tests for all 4 without
+    // branches, then one EdgeFunction per needed query (act: 4 query bits; an unreached u —
+    // a pull may read one — is never Needed).
     __device__ static uint32_t relax(uint32_t* p, const uint32_t (&u)[G], const uint32_t (&c)[G], const Arg& w,
                                      uint32_t act, uint32_t& n_edges, uint32_t& n_upd, uint32_t*) {
-        if (!act || u[0] == O::INIT) return 0u;  // (a pull may read an unreached u)
-        ++n_edges;
-        uint32_t cand;
+        uint32_t cand[G], ok = 0, ch = 0;
+#pragma unroll
+        for (int i = 0; i < G; ++i) ok |= (uint32_t)(u[i] != O::INIT) << i;
+        ok &= act;
+        n_edges += __popc(ok);
         if constexpr (VIT) {
-            cand = vit_div(u[0], w);
+            vit_div4(u, w, cand);
         } else {
-            cand = O::ext(u[0], w);
+#pragma unroll
+            for (int i = 0; i < G; ++i) cand[i] = O::ext(u[i], w);
         }
-        if (!O::better(cand, c[0])) return 0u;  // Needed(e(u,v))
-        O::edge_fn(p, cand);                  // EdgeFunction
-        ++n_upd;
-        return 1u;
+#pragma unroll
+        for (int i = 0; i < G; ++i) ch |= (uint32_t)O::better(cand[i], c[i]) << i;  // Needed(e(u,v))
+        ch &= ok;
+        if (!ch) return 0u;
+#pragma unroll
+        for (int i = 0; i < G; ++i)
+            if ((ch >> i) & 1u) O::edge_fn(p + i, cand[i]);  // EdgeFunction
+        n_upd += __popc(ch);
+        return ch;
     }
 };
 

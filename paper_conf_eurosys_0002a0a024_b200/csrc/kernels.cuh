@@ -62,6 +62,25 @@ __device__ __forceinline__ uint32_t vit_div(uint32_t a, const VitArg& A) {
     return __float_as_uint(y);
 }
 
+// four quotients of one edge (a batch row's 16 B group): the fast path for all four, one
+// warp-divergent branch to __fdiv_rn only when some lane falls outside it
+__device__ __forceinline__ void vit_div4(const uint32_t (&a)[4], const VitArg& A, uint32_t (&out)[4]) {
+    const float b = __uint2float_rn(A.w);
+    bool slow = A.r == 0.0f;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+        const float x = __uint_as_float(a[i]);
+        const float q = __fmul_rn(x, A.r);
+        const float e = __fmaf_rn(-q, b, x);
+        out[i] = __float_as_uint(__fmaf_rn(e, A.r, q));
+        slow |= !(x >= 0x1p-64f) && a[i] != 0u;  // (0 / w = 0 on the fast path too)
+    }
+    if (slow) {
+#pragma unroll
+        for (int i = 0; i < 4; ++i) out[i] = vit_div(a[i], A);
+    }
+}
+
 template <> struct Op<CG_BFS> {
     static constexpr uint32_t INIT = 0xffffffffu, SRC = 0u;
     __device__ static uint32_t ext(uint32_t a, uint32_t) { return a + 1u; }
