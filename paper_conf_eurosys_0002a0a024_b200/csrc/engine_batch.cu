@@ -766,6 +766,9 @@ __device__ __forceinline__ uint32_t first_entry(const BParams& P, uint32_t count
     return lo + 31 - __clz(__ballot_sync(FULL, le));
 }
 
+template <class L>  // 128 B rows (RW = 32): one window buffer, so 16 warps' buffers fit in shared memory
+constexpr bool xs_double() { return L::RW <= 16; }
+
 // S2 over the compacted list: the iteration's E list edges split evenly over all warps; a warp
 // slides 32-entry windows (a hub row is shared by as many warps and CTAs as needed).  Windows
 // are prefetched one ahead: while window i's edges run, window i+1's source rows are already
@@ -800,6 +803,7 @@ __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, ui
         }
         cp_async_commit();
     };
+    constexpr bool DB = xs_double<L>();  // next window's rows copied while this one runs
     uint32_t i = first_entry(P, count, e0), e = e0;
     uint32_t cv, coff, cmask, nv, noff, nmask;
     list_load(i, cv, coff, cmask);
@@ -814,20 +818,20 @@ __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, ui
         uint32_t nbase = 0, mv = 0, moff = E, mmask = 0;
         if (more) {
             nbase = i + 32 + lane < count ? __ldg(g.ptr + nv) - noff : 0u;
-            rows_async(xs + (buf ^ 1) * 32 * RW, nv, i + 32);
+            if constexpr (DB) rows_async(xs + (buf ^ 1) * 32 * RW, nv, i + 32);
             list_load(i + 64, mv, moff, mmask);
-            cp_async_wait<1>();  // this window's rows (the next window's may still fly)
-        } else {
-            cp_async_wait<0>();
         }
+        if (DB && more) cp_async_wait<1>();  // this window's rows (the next window's may still fly)
+        else cp_async_wait<0>();
         __syncwarp();
         window_edges<KIND, PACKED, L>(P, g, xs + buf * 32 * RW, vs, coff, cbase, cmask, e, ehi, set_bits, fresh,
                                       n_edges, n_upd, n_read);
         __syncwarp();  // every lane is done with this window's rows before they are overwritten
         if (!more) break;
+        if constexpr (!DB) rows_async(xs, nv, i + 32);
         e = ehi;
         i += 32;
-        buf ^= 1;
+        if constexpr (DB) buf ^= 1;
         cv = nv;
         coff = noff;
         cmask = nmask;
@@ -1000,8 +1004,11 @@ __device__ void transpose_out(const BParams& P, uint32_t* dst, int q0, int nq, u
     }
 }
 
-template <class L>  // per warp, 16 B aligned: two 32-row windows (S2) or the padded transpose tile
-constexpr uint32_t xs_words() { return 2 * 32 * L::RW > ((32 * (L::RW + 1) + 3) & ~3u) ? 2 * 32 * L::RW : ((32 * (L::RW + 1) + 3) & ~3u); }
+template <class L>  // per warp, 16 B aligned: one or two 32-row windows (S2) or the padded transpose tile
+constexpr uint32_t xs_words() {
+    return (xs_double<L>() ? 2 : 1) * 32 * L::RW > ((32 * (L::RW + 1) + 3) & ~3u) ? (xs_double<L>() ? 2 : 1) * 32 * L::RW
+                                                                                 : ((32 * (L::RW + 1) + 3) & ~3u);
+}
 template <class L>
 constexpr uint32_t vs_words() { return S_PIPE * 32 * L::RW; }
 
