@@ -634,12 +634,15 @@ __device__ __forceinline__ void window_edges(const BParams& P, const GraphView& 
     uint32_t ek[EA];               // their window row (NONE: no edge / inactive row)
     uint32_t sd[S], sw[S], sk[S];  // requested chunks (slot = chunk % S): destination, weight, window row
 
+    // the window row of each lane's edge t = cs + lane: rows starting at or before cs (one
+    // ballot) plus the rows starting in (cs, t] (one warp OR of start bits) — no dependent
+    // shuffle search; the list holds rows with edges only, so row starts are distinct
     auto fetch = [&](uint32_t c, EdgeWord<PACKED>& wd, uint32_t& kout) {
-        const uint32_t t = e + c * 32 + lane;
-        uint32_t kk = 0;
-#pragma unroll
-        for (uint32_t st = 16; st > 0; st >>= 1)
-            if (__shfl_sync(FULL, off, kk + st) <= t) kk += st;
+        const uint32_t cs = e + c * 32, t = cs + lane;
+        const uint32_t below = __popc(__ballot_sync(FULL, off <= cs));  // >= 1: row 0 starts at or before e
+        const uint32_t rel = off - cs;
+        const uint32_t starts = __reduce_or_sync(FULL, (rel - 1u < 31u) ? (1u << rel) : 0u);
+        const uint32_t kk = below - 1u + __popc(starts & ((2u << lane) - 1u));
         const uint32_t mk = __shfl_sync(FULL, mask, kk);
         const uint32_t a = __shfl_sync(FULL, base, kk) + t;
         const bool ok = t < ehi && mk != 0u;
