@@ -961,12 +961,12 @@ __device__ void transpose_out(const BParams& P, uint32_t* dst, int q0, int nq, u
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t gw = blockIdx.x * BW + (threadIdx.x >> 5);
     const uint32_t NW = gridDim.x * BW;
-    for (uint32_t v0 = gw * 32; v0 < P.n; v0 += NW * 32 * TU) {
+    for (uint32_t v0 = gw * 32 * TU; v0 < P.n; v0 += NW * 32 * TU) {  // TU adjacent tiles: 128 TU B runs per query
         uint4 x4[V4 ? TU * NC : 1];
         uint32_t x1[V4 ? 1 : TU * NC];
 #pragma unroll
         for (int t = 0; t < TU; ++t) {
-            const uint32_t vt = v0 + t * NW * 32;
+            const uint32_t vt = v0 + t * 32;
 #pragma unroll
             for (int r = 0; r < NC; ++r) {
                 const uint32_t f = r * 32 + lane;  // chunk f of the tile's 32 rows
@@ -981,7 +981,7 @@ __device__ void transpose_out(const BParams& P, uint32_t* dst, int q0, int nq, u
         }
 #pragma unroll
         for (int t = 0; t < TU; ++t) {
-            const uint32_t vt = v0 + t * NW * 32;
+            const uint32_t vt = v0 + t * 32;
             if (vt >= P.n) break;
             __syncwarp();
 #pragma unroll
@@ -1037,7 +1037,14 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
     for (int q0 = 0; q0 < P.n_src; q0 += Q) {
         const int nq = min(Q, P.n_src - q0);
         // Alg 3 l.4, l.6 for every query of the batch; masks cleared
-        for (uint64_t i = tid; i < (uint64_t)P.n * RW; i += nthreads) P.V[i] = InitOf<L>::at(i);
+        if constexpr (RW % 4 == 0 && !InitOf<L>::ALL_ACTIVE) {  // 16 B stores
+            const uint32_t iw = L::init_word();
+            const uint4 x = make_uint4(iw, iw, iw, iw);
+            uint4* V4 = reinterpret_cast<uint4*>(P.V);
+            for (uint64_t i = tid; i < (uint64_t)P.n * (RW / 4); i += nthreads) V4[i] = x;
+        } else {
+            for (uint64_t i = tid; i < (uint64_t)P.n * RW; i += nthreads) P.V[i] = InitOf<L>::at(i);
+        }
         for (uint64_t v = tid; v < P.n; v += nthreads) P.M[v] = InitOf<L>::ALL_ACTIVE ? 1u : 0u;
         grid_sync(P.ctrl, epoch);
         for (int b = 0; b < nq && !InitOf<L>::ALL_ACTIVE; ++b) {
