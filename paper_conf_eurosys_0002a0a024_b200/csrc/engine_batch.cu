@@ -146,9 +146,13 @@ struct Lanes16 {
     static constexpr uint32_t INF16 = 0x7c00u, LIMIT = 0x68006800u;  // +inf; 2048.0 in both lanes
     static constexpr uint32_t INIT16 = MAXK ? 0u : INF16, SRC16 = MAXK ? INF16 : 0u;
     __device__ static uint32_t init_word() { return INIT16 * 0x10001u; }
+    // lane j as a u32: values are integers in [0, 2048) (or +inf), so the binary16 pattern
+    // decodes with integer ops — significand with its hidden bit, shifted by 25 - biased
+    // exponent (0 -> 0 falls out of the shift) — instead of two quarter-rate conversions
     __device__ static uint32_t decode(uint32_t x, uint32_t j) {
         const uint32_t h = (x >> (16 * j)) & 0xffffu;
-        return h == INF16 ? 0xffffffffu : (uint32_t)__half2float(__ushort_as_half((unsigned short)h));
+        const uint32_t k = ((h & 0x3ffu) | 0x400u) >> min(25u - (h >> 10), 31u);
+        return h == INF16 ? 0xffffffffu : k;
     }
     __device__ static uint32_t bits2(uint32_t m) { return ((m >> 15) & 1u) | ((m >> 30) & 2u); }  // 0xffff lanes -> 2 bits
     __device__ static uint32_t halves2(uint32_t b) { return ((b & 1u) ? 0xffffu : 0u) | ((b & 2u) ? 0xffff0000u : 0u); }
@@ -948,58 +952,79 @@ __device__ __forceinline__ uint32_t value_of(const uint32_t* V, uint32_t v, uint
     return L::decode(ld_cg(V + (size_t)v * L::RW + q / L::QPW), q % L::QPW);
 }
 
-// rows -> dst[(q0+q)*n + v] for q < nq, 32 vertices per warp through shared memory: the 32
-// rows are read with 16 B loads (coalesced), each lane decodes its vertex's Q values, and every
-// query's 32 values leave as one 128 B streaming store.  A warp keeps TU tiles' loads in flight
-// (registers) before it stages them one at a time through its padded shared tile.
+#ifndef CGB_TSTORE
+#define CGB_TSTORE 0
+#endif
+__device__ __forceinline__ void tstore(uint32_t* p, uint32_t x) {
+    if (CGB_TSTORE == 0) __stcs(p, x);
+    else if (CGB_TSTORE == 1) *p = x;
+    else __stcg(p, x);
+}
+
+// rows -> dst[(q0+q)*n + v] for q < nq, 32 vertices (a tile) per warp through shared memory:
+// each lane decodes its vertex's Q values and every query's 32 values leave as one 128 B
+// streaming store.  16 B-row layouts stage tiles two ahead in the warp's (then idle) S2 row
+// ring `vs` with cp.async, so the row reads of later tiles overlap this tile's stores; the
+// staged tile is copied into the padded tile in xs (conflict-free column reads).
 template <class L>
-__device__ void transpose_out(const BParams& P, uint32_t* dst, int q0, int nq, uint32_t* xs) {
+__device__ void transpose_out(const BParams& P, uint32_t* dst, int q0, int nq, uint32_t* xs, uint32_t* vs) {
     constexpr int RW = L::RW;
-    constexpr bool V4 = RW % 4 == 0;
-    constexpr int NC = V4 ? RW / 4 : RW;  // loads per lane per tile
-    constexpr int TU = NC >= 8 ? 2 : 4;  // <= 16 x 16 B in flight per lane
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t gw = blockIdx.x * BW + (threadIdx.x >> 5);
     const uint32_t NW = gridDim.x * BW;
-    for (uint32_t v0 = gw * 32 * TU; v0 < P.n; v0 += NW * 32 * TU) {  // TU adjacent tiles: 128 TU B runs per query
-        uint4 x4[V4 ? TU * NC : 1];
-        uint32_t x1[V4 ? 1 : TU * NC];
+    const uint32_t T = (P.n + 31) / 32;  // tiles
+    if constexpr (RW % 4 == 0) {
+        constexpr int NC = RW / 4;          // 16 B pieces per lane per tile
+        constexpr uint32_t TW = 32 * RW;    // staged words per tile
+        static_assert(2 * TW <= S_PIPE * 32 * RW, "two staged tiles fit the row ring");
+        auto stage = [&](uint32_t tile, int slot) {
+            if (tile < T) {
 #pragma unroll
-        for (int t = 0; t < TU; ++t) {
-            const uint32_t vt = v0 + t * 32;
-#pragma unroll
-            for (int r = 0; r < NC; ++r) {
-                const uint32_t f = r * 32 + lane;  // chunk f of the tile's 32 rows
-                const uint32_t v = vt + f / NC, c = f % NC;
-                if constexpr (V4) {
-                    x4[t * NC + r] = v < P.n ? __ldcg(reinterpret_cast<const uint4*>(P.V + (size_t)v * RW) + c)
-                                             : make_uint4(0, 0, 0, 0);
-                } else {
-                    x1[t * NC + r] = v < P.n ? __ldcg(P.V + (size_t)v * RW + c) : 0u;
+                for (int r = 0; r < NC; ++r) {
+                    const uint32_t f = r * 32 + lane, row = f / NC, c = f % NC;
+                    const uint32_t v = tile * 32 + row;
+                    if (v < P.n) cp_async16_cg(vs + slot * TW + row * RW + 4 * c, P.V + (size_t)v * RW + 4 * c);
                 }
             }
+            cp_async_commit();
+        };
+        stage(gw, 0);
+        stage(gw + NW, 1);
+        int slot = 0;
+        for (uint32_t tile = gw; tile < T; tile += NW) {
+            cp_async_wait<1>();
+            __syncwarp();
+#pragma unroll
+            for (int r = 0; r < NC; ++r) {
+                const uint32_t f = r * 32 + lane, row = f / NC, c = f % NC;
+                const uint4 x = *reinterpret_cast<const uint4*>(vs + slot * TW + row * RW + 4 * c);
+                uint32_t* d = xs + row * (RW + 1) + 4 * c;
+                d[0] = x.x;
+                d[1] = x.y;
+                d[2] = x.z;
+                d[3] = x.w;
+            }
+            __syncwarp();
+            stage(tile + 2 * NW, slot);  // refill the slot just read
+            const uint32_t v = tile * 32 + lane;
+            if (v < P.n)
+                for (int q = 0; q < nq; ++q)
+                    tstore(dst + (size_t)(q0 + q) * P.n + v, L::decode(xs[lane * (RW + 1) + q / L::QPW], q % L::QPW));
+            __syncwarp();  // xs is rewritten by the next tile
+            slot ^= 1;
         }
-#pragma unroll
-        for (int t = 0; t < TU; ++t) {
-            const uint32_t vt = v0 + t * 32;
-            if (vt >= P.n) break;
+        cp_async_wait<0>();
+    } else {
+        for (uint32_t tile = gw; tile < T; tile += NW) {
             __syncwarp();
 #pragma unroll
-            for (int r = 0; r < NC; ++r) {
+            for (int r = 0; r < RW; ++r) {
                 const uint32_t f = r * 32 + lane;
-                if constexpr (V4) {
-                    uint32_t* d = xs + (f / NC) * (RW + 1) + 4 * (f % NC);
-                    const uint4 x = x4[t * NC + r];
-                    d[0] = x.x;
-                    d[1] = x.y;
-                    d[2] = x.z;
-                    d[3] = x.w;
-                } else {
-                    xs[(f / NC) * (RW + 1) + f % NC] = x1[t * NC + r];
-                }
+                const uint32_t v = tile * 32 + f / RW;
+                xs[(f / RW) * (RW + 1) + f % RW] = v < P.n ? __ldcg(P.V + (size_t)v * RW + f % RW) : 0u;
             }
             __syncwarp();
-            const uint32_t v = vt + lane;
+            const uint32_t v = tile * 32 + lane;
             if (v < P.n)
                 for (int q = 0; q < nq; ++q)
                     __stcs(dst + (size_t)(q0 + q) * P.n + v, L::decode(xs[lane * (RW + 1) + q / L::QPW], q % L::QPW));
@@ -1137,7 +1162,7 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
                 n_edges = n_upd = n_read = 0;
                 iters = 0;
                 if (phase == 1) {
-                    if (P.p1) transpose_out<L>(P, P.p1, q0, nq, xs);
+                    if (P.p1) transpose_out<L>(P, P.p1, q0, nq, xs, vs);
                     if (P.stats) {  // impacted per query (Alg 3 l.15); the thread's query q is fixed
                         const uint32_t q = (uint32_t)(tid % Q);
                         const uint32_t init = L::decode(L::init_word(), 0);
@@ -1174,7 +1199,7 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
             }
         }
         if (kt && q0 == 0) kt[2] = global_ns();
-        transpose_out<L>(P, P.out, q0, nq, xs);
+        transpose_out<L>(P, P.out, q0, nq, xs, vs);
         if (P.stats) {  // reached / precise per query (the thread's query q is fixed)
             const uint32_t q = (uint32_t)(tid % Q);
             const uint32_t sb = ((int)q < nq && P.srcs) ? __ldg(P.srcs + q0 + q) : 0xffffffffu;
