@@ -503,29 +503,37 @@ __device__ __forceinline__ void span_loads(const BParams& P, const GraphView& g,
     }
 }
 
+#ifndef CGB_S1H
+#define CGB_S1H 2
+#endif
 __device__ void compact_masks(const BParams& P, const GraphView& g, unsigned long long* cnt_slot,
                               unsigned long long* act_slot, uint32_t* sm) {
-    // One pass: the CTA's word range is taken in rounds of BW half-spans (16 words = 512
-    // vertices per warp); a round's masks and degrees stay in registers while the CTA reserves
-    // its list range (one 64-bit atomicAdd per round), then the entries are written and the
-    // masks consumed.  List order is vertex order within a round; S2 needs only that the edge
-    // offsets ascend with the list index, which the packed (count, edges) reservation gives.
+    // One pass: the CTA's word range is taken in rounds of BW x H half-spans (H x 16 words =
+    // H x 512 vertices per warp, all loads of a round issued together); a round's masks and
+    // degrees stay in registers while the CTA reserves its list range (one 64-bit atomicAdd
+    // per round), then the entries are written and the masks consumed.  List order is vertex
+    // order within a round; S2 needs only that the edge offsets ascend with the list index,
+    // which the packed (count, edges) reservation gives.
+    constexpr int H = CGB_S1H;
     const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const uint64_t W = P.words;
     const uint32_t w0 = (uint32_t)(W * blockIdx.x / gridDim.x), w1 = (uint32_t)(W * (blockIdx.x + 1) / gridDim.x);
     const uint32_t lt = (1u << lane) - 1u;
     uint32_t active = 0;
-    for (uint32_t r0 = w0; r0 < w1; r0 += BW * 16) {
-        const uint32_t g0 = r0 + warp * 16;
-        uint32_t mv[16], dg[16];
-        span_loads(P, g, g0, w1, 0, mv, dg);
+    for (uint32_t r0 = w0; r0 < w1; r0 += BW * 16 * H) {
+        const uint32_t g0 = r0 + warp * 16 * H;
+        uint32_t mv[H][16], dg[H][16];
+#pragma unroll
+        for (int h = 0; h < H; ++h) span_loads(P, g, g0, w1, h, mv[h], dg[h]);
         uint32_t cnt = 0, edges = 0;
 #pragma unroll
-        for (int j = 0; j < 16; ++j) {
-            active += mv[j] != 0u;
-            cnt += dg[j] != 0u;
-            edges += dg[j];
-        }
+        for (int h = 0; h < H; ++h)
+#pragma unroll
+            for (int j = 0; j < 16; ++j) {
+                active += mv[h][j] != 0u;
+                cnt += dg[h][j] != 0u;
+                edges += dg[h][j];
+            }
         for (int o = 16; o > 0; o >>= 1) {
             cnt += __shfl_xor_sync(FULL, cnt, o);
             edges += __shfl_xor_sync(FULL, edges, o);
@@ -554,26 +562,28 @@ __device__ void compact_masks(const BParams& P, const GraphView& g, unsigned lon
         uint32_t eb = sm[2 * BW + 1] + sm[BW + warp];
         __syncthreads();  // sm is rewritten by the next round
 #pragma unroll
-        for (int j = 0; j < 16; ++j) {
-            const uint32_t v = (g0 + j) * 32 + lane;
-            if (mv[j]) P.M[v] = 0u;  // consumed
-            const uint32_t d = dg[j];
-            uint32_t incl = d;
+        for (int h = 0; h < H; ++h)
 #pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const uint32_t y = __shfl_up_sync(FULL, incl, o);
-                if (lane >= (uint32_t)o) incl += y;
+            for (int j = 0; j < 16; ++j) {
+                const uint32_t v = (g0 + h * 16 + j) * 32 + lane;
+                if (mv[h][j]) P.M[v] = 0u;  // consumed
+                const uint32_t d = dg[h][j];
+                uint32_t incl = d;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const uint32_t y = __shfl_up_sync(FULL, incl, o);
+                    if (lane >= (uint32_t)o) incl += y;
+                }
+                const uint32_t bal = __ballot_sync(FULL, d != 0);
+                if (d) {
+                    const uint32_t i = pos + __popc(bal & lt);
+                    P.lv[i] = v;
+                    P.lo[i] = eb + incl - d;
+                    P.lm[i] = mv[h][j];
+                }
+                pos += __popc(bal);
+                eb += __shfl_sync(FULL, incl, 31);
             }
-            const uint32_t bal = __ballot_sync(FULL, d != 0);
-            if (d) {
-                const uint32_t i = pos + __popc(bal & lt);
-                P.lv[i] = v;
-                P.lo[i] = eb + incl - d;
-                P.lm[i] = mv[j];
-            }
-            pos += __popc(bal);
-            eb += __shfl_sync(FULL, incl, 31);
-        }
     }
     for (int o = 16; o > 0; o >>= 1) active += __shfl_xor_sync(FULL, active, o);
     if (lane == 0 && active) atomicAdd(act_slot, (unsigned long long)active);
