@@ -69,7 +69,6 @@ struct BParams {
     uint32_t K, KP;             // hubs in HB; row stride 2*KP (KP = K rounded up to a multiple of 4)
     int reduced;                // phase 2 starts with the certificate-driven pull (NEXT-1)
     uint32_t fresh;             // bit p-1: phase p pre-reads values from L2 instead of L1
-    int implicit;               // phase 2's first sweep walks the implicit all-vertex list
     unsigned long long* trace;  // nullable: per iteration {t_start, t_s1, t_s2, phase<<62|q0<<32|listed, active<<32|edges}
     uint32_t trace_cap;
 };
@@ -634,7 +633,7 @@ template <class L> struct RowCopy {
 template <int KIND, bool PACKED, class L>
 __device__ __forceinline__ void window_edges(const BParams& P, const GraphView& g, const uint32_t* xs, uint32_t* vs,
                                              uint32_t off, uint32_t base, uint32_t mask, uint32_t e, uint32_t ehi,
-                                             bool set_bits, bool fresh, bool dup, uint32_t& n_edges, uint32_t& n_upd,
+                                             bool set_bits, bool fresh, uint32_t& n_edges, uint32_t& n_upd,
                                              uint32_t& n_read) {
     constexpr int S = S_PIPE, EA = E_AHEAD, RW = L::RW;
     static_assert(EA % S == 0 && EA >= S, "E_AHEAD must be a multiple of S_PIPE");
@@ -652,22 +651,12 @@ __device__ __forceinline__ void window_edges(const BParams& P, const GraphView& 
     // the window row of each lane's edge t = cs + lane: rows starting at or before cs (one
     // ballot) plus the rows starting in (cs, t] (one warp OR of start bits) — no dependent
     // shuffle search; the list holds rows with edges only, so row starts are distinct
-    // (dup: rows without edges share their successor's start — the implicit list — so the
-    // last row starting at or before t is found by a 5-step shuffle search instead)
     auto fetch = [&](uint32_t c, EdgeWord<PACKED>& wd, uint32_t& kout) {
         const uint32_t cs = e + c * 32, t = cs + lane;
-        uint32_t kk;
-        if (!dup) {
-            const uint32_t below = __popc(__ballot_sync(FULL, off <= cs));  // >= 1: row 0 starts at or before e
-            const uint32_t rel = off - cs;
-            const uint32_t starts = __reduce_or_sync(FULL, (rel - 1u < 31u) ? (1u << rel) : 0u);
-            kk = below - 1u + __popc(starts & ((2u << lane) - 1u));
-        } else {
-            kk = 0;
-#pragma unroll
-            for (uint32_t st = 16; st > 0; st >>= 1)
-                if (__shfl_sync(FULL, off, kk + st) <= t) kk += st;
-        }
+        const uint32_t below = __popc(__ballot_sync(FULL, off <= cs));  // >= 1: row 0 starts at or before e
+        const uint32_t rel = off - cs;
+        const uint32_t starts = __reduce_or_sync(FULL, (rel - 1u < 31u) ? (1u << rel) : 0u);
+        const uint32_t kk = below - 1u + __popc(starts & ((2u << lane) - 1u));
         const uint32_t mk = __shfl_sync(FULL, mask, kk);
         const uint32_t a = __shfl_sync(FULL, base, kk) + t;
         const bool ok = t < ehi && mk != 0u;
@@ -777,20 +766,20 @@ __device__ __forceinline__ void load_rows(const BParams& P, uint32_t* xs, uint32
 }
 
 // first list entry of the warp's edge range: 32-ary search over the list's edge offsets
-__device__ __forceinline__ uint32_t first_entry(const uint32_t* offs, uint32_t count, uint32_t e0) {
+__device__ __forceinline__ uint32_t first_entry(const BParams& P, uint32_t count, uint32_t e0) {
     const uint32_t lane = threadIdx.x & 31;
     uint32_t lo = 0, hi = count;
     while (hi - lo > 32) {
         const uint32_t step = (hi - lo + 31) / 32;
         const uint32_t p = lo + lane * step;
-        const bool le = p < hi && ld_cg(offs + p) <= e0;
+        const bool le = p < hi && ld_cg(P.lo + p) <= e0;
         const uint32_t k = 31 - __clz(__ballot_sync(FULL, le));
         const uint32_t nlo = lo + k * step;
         hi = min(hi, nlo + step);
         lo = nlo;
     }
     const uint32_t p = lo + lane;
-    const bool le = p < hi && ld_cg(offs + p) <= e0;
+    const bool le = p < hi && ld_cg(P.lo + p) <= e0;
     return lo + 31 - __clz(__ballot_sync(FULL, le));
 }
 
@@ -802,12 +791,8 @@ constexpr bool xs_double() { return L::RW <= 16; }
 // are prefetched one ahead: while window i's edges run, window i+1's source rows are already
 // being copied (cp.async) into the other half of xs and window i+2's list entries are loading.
 template <int KIND, bool PACKED, class L>
-//
-// implicit: the list is every vertex in id order with its CSR offsets (count = n, E = m; no S1):
-// Alg 3 l.15's first phase-2 frontier, whose query masks are the window rows' reached lanes.
 __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, uint32_t E, uint32_t* xs, uint32_t* vs,
-                        bool set_bits, bool fresh, uint32_t& n_edges, uint32_t& n_upd, uint32_t& n_read,
-                        bool implicit = false) {
+                        bool set_bits, bool fresh, uint32_t& n_edges, uint32_t& n_upd, uint32_t& n_read) {
     constexpr int RW = L::RW;
     using RC = RowCopy<L>;
     const uint32_t lane = threadIdx.x & 31;
@@ -821,14 +806,9 @@ __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, ui
         off = E;
         mask = 0;
         if (idx < count) {
-            if (implicit) {
-                v = idx;
-                off = __ldg(g.ptr + idx);
-            } else {
-                v = ld_cg(P.lv + idx);
-                off = ld_cg(P.lo + idx);
-                mask = ld_cg(P.lm + idx);
-            }
+            v = ld_cg(P.lv + idx);
+            off = ld_cg(P.lo + idx);
+            mask = ld_cg(P.lm + idx);
         }
     };
     auto rows_async = [&](uint32_t* buf, uint32_t v, uint32_t i0) {  // the window's 32 rows -> buf
@@ -841,10 +821,10 @@ __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, ui
         cp_async_commit();
     };
     constexpr bool DB = xs_double<L>();  // next window's rows copied while this one runs
-    uint32_t i = first_entry(implicit ? g.ptr : P.lo, count, e0), e = e0;
+    uint32_t i = first_entry(P, count, e0), e = e0;
     uint32_t cv, coff, cmask, nv, noff, nmask;
     list_load(i, cv, coff, cmask);
-    uint32_t cbase = i + lane < count && !implicit ? __ldg(g.ptr + cv) - coff : 0u;
+    uint32_t cbase = i + lane < count ? __ldg(g.ptr + cv) - coff : 0u;
     rows_async(xs, cv, i);
     list_load(i + 32, nv, noff, nmask);
     uint32_t buf = 0;
@@ -854,23 +834,15 @@ __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, ui
         const bool more = ehi < e1;
         uint32_t nbase = 0, mv = 0, moff = E, mmask = 0;
         if (more) {
-            nbase = i + 32 + lane < count && !implicit ? __ldg(g.ptr + nv) - noff : 0u;
+            nbase = i + 32 + lane < count ? __ldg(g.ptr + nv) - noff : 0u;
             if constexpr (DB) rows_async(xs + (buf ^ 1) * 32 * RW, nv, i + 32);
             list_load(i + 64, mv, moff, mmask);
         }
         if (DB && more) cp_async_wait<1>();  // this window's rows (the next window's may still fly)
         else cp_async_wait<0>();
         __syncwarp();
-        if (implicit) {  // Alg 3 l.15: the row's queries with Val != InitVal
-            cmask = 0;
-            if (i + lane < count) {
-                const uint32_t* r = xs + buf * 32 * RW + lane * RW;
-#pragma unroll
-                for (int w = 0; w < RW; ++w) cmask |= L::live(r[w]) << (w * L::QPW);
-            }
-        }
         window_edges<KIND, PACKED, L>(P, g, xs + buf * 32 * RW, vs, coff, cbase, cmask, e, ehi, set_bits, fresh,
-                                      implicit, n_edges, n_upd, n_read);
+                                      n_edges, n_upd, n_read);
         __syncwarp();  // every lane is done with this window's rows before they are overwritten
         if (!more) break;
         if constexpr (!DB) rows_async(xs, nv, i + 32);
@@ -902,7 +874,7 @@ __device__ void relax_pull(const BParams& P, uint32_t count, uint32_t E, uint32_
     const uint64_t NW = (uint64_t)gridDim.x * BW;
     const uint32_t e0 = (uint32_t)((uint64_t)E * gw / NW), e1 = (uint32_t)((uint64_t)E * (gw + 1) / NW);
     if (e0 >= e1) return;
-    uint32_t i = first_entry(P.lo, count, e0), e = e0;
+    uint32_t i = first_entry(P, count, e0), e = e0;
     for (;;) {
         const uint32_t idx = i + lane;
         uint32_t off = E, base = 0, v = 0, mask = 0;
@@ -1157,12 +1129,7 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
             }
             const unsigned long long t_s0 = (P.trace && tid == 0) ? global_ns() : 0ull;
             const int mode = pull ? F_UNCERT : predicate ? F_IMPACTED : bits ? F_BITS : F_MASKS;
-            // the first phase-2 frontier (l.15) is nearly every vertex with edges: S2 walks the
-            // implicit list (all vertices, CSR offsets) and takes the masks from the rows — no
-            // mark pass, no compaction (counters-on runs keep the explicit list for the stats)
-            const bool impl = mode == F_IMPACTED && P.implicit && !P.stats;
-            if (impl) {
-            } else if (mode == F_BITS) {
+            if (mode == F_BITS) {
                 compact_bits(P, g, ctr + CT_LIST, ctr + CT_ACTIVE, sm_cnt);
             } else {
                 if (mode != F_MASKS) {  // impacted (l.15) / uncertified (NEXT-1) queries into M
@@ -1171,17 +1138,10 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
                 }
                 compact_masks(P, pull ? P.R : g, ctr + CT_LIST, ctr + CT_ACTIVE, sm_cnt);
             }
-            if (!impl) grid_sync(P.ctrl, epoch);
+            grid_sync(P.ctrl, epoch);
             ++ring;
-            uint32_t count, E;
-            if (impl) {
-                count = P.n;
-                E = __ldg(g.ptr + P.n);
-            } else {
-                const unsigned long long ce = ld_cg64(ctr + CT_LIST);
-                count = (uint32_t)(ce >> 32);
-                E = (uint32_t)ce;
-            }
+            const unsigned long long ce = ld_cg64(ctr + CT_LIST);
+            const uint32_t count = (uint32_t)(ce >> 32), E = (uint32_t)ce;
             const uint32_t tr = ring - 1;
             if (P.trace && tid == 0 && tr + 1 < P.trace_cap) {
                 unsigned long long* t = P.trace + 5ull * tr;
@@ -1238,7 +1198,7 @@ __global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
                 // small frontier: its S2 sets frontier bits (few reds) and the next S1 reads the
                 // bitmap; large frontier: no bitmap reds (they contend in L2), the next S1 scans M
                 bits = E < P.bits_below;  // at most E vertices change
-                relax_b<KIND, PACKED, L>(P, g, count, E, xs, vs, bits, fresh, n_edges, n_upd, n_read, impl);
+                relax_b<KIND, PACKED, L>(P, g, count, E, xs, vs, bits, fresh, n_edges, n_upd, n_read);
                 predicate = false;
             }
             grid_sync(P.ctrl, epoch);
@@ -1399,8 +1359,6 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
         P.bits_below = e ? (uint32_t)strtoul(e, nullptr, 10) : G.n / 256;
         const char* f = getenv("CG_FRESH");
         P.fresh = f ? (uint32_t)strtoul(f, nullptr, 10) : 0u;
-        const char* im = getenv("CG_IMPLICIT");
-        P.implicit = im ? atoi(im) : 1;
     }
     CGB_CUDA(cudaMemsetAsync(w.bitmap.get(), 0, w.bitmap.bytes(), s));
     CGB_CUDA(cudaMemsetAsync(w.ctrl.get(), 0, w.ctrl.bytes(), s));
