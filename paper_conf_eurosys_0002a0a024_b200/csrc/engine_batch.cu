@@ -1358,7 +1358,7 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
         const char* e = getenv("CG_BITS_BELOW");
         P.bits_below = e ? (uint32_t)strtoul(e, nullptr, 10) : G.n / 256;
         const char* f = getenv("CG_FRESH");
-        P.fresh = f ? (uint32_t)strtoul(f, nullptr, 10) : 0u;
+        P.fresh = f ? (uint32_t)strtoul(f, nullptr, 10) : 2u;  // phase 2 gathers bypass L1 (measured +1 %; L1 hit rate ~4 %)
     }
     CGB_CUDA(cudaMemsetAsync(w.bitmap.get(), 0, w.bitmap.bytes(), s));
     CGB_CUDA(cudaMemsetAsync(w.ctrl.get(), 0, w.ctrl.bytes(), s));
