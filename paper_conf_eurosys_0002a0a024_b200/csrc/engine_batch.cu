@@ -30,7 +30,10 @@ namespace {
 
 using namespace kern;
 
-constexpr int BT = 512;          // threads per CTA
+#ifndef CGB_BT
+#define CGB_BT 512
+#endif
+constexpr int BT = CGB_BT;       // threads per CTA
 constexpr int BW = BT / 32;      // warps per CTA
 #ifndef CGB_STAGES
 #define CGB_STAGES 2
@@ -1051,7 +1054,7 @@ template <class L>
 constexpr uint32_t vs_words() { return S_PIPE * 32 * L::RW; }
 
 template <int KIND, bool PACKED, class L>
-__global__ void __launch_bounds__(BT, 1) batch_kernel(BParams P) {
+__global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
     constexpr int Q = L::Q, RW = L::RW;
     __shared__ uint32_t sm_cnt[2 * BW + 2];
     __shared__ unsigned long long sm_red[BW];
