@@ -149,14 +149,15 @@ __global__ void k_connectivity(uint32_t n, GraphView g, uint32_t dbits, int kind
 }
 
 // ---------------------------------------------------------------- a7: compaction
+// (inv: count / scatter the UNflagged edges — G minus the CG, phase 2's first sweep)
 __global__ void k_row_count(uint32_t n, const uint32_t* __restrict__ ptr, const uint8_t* __restrict__ flags,
-                            uint32_t* __restrict__ cnt) {
+                            uint32_t* __restrict__ cnt, int inv = 0) {
     const uint32_t lane = threadIdx.x & 31;
     const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
     for (uint64_t u = blockIdx.x * (uint64_t)(blockDim.x / 32) + (threadIdx.x >> 5); u <= n; u += nw) {
         if (u == n) { if (lane == 0) cnt[n] = 0; continue; }
         uint32_t c = 0;
-        for (uint32_t e = ptr[u] + lane; e < ptr[u + 1]; e += 32) c += flags[e] != 0;
+        for (uint32_t e = ptr[u] + lane; e < ptr[u + 1]; e += 32) c += (flags[e] != 0) != (inv != 0);
         for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(FULLM, c, o);
         if (lane == 0) cnt[u] = c;
     }
@@ -164,7 +165,8 @@ __global__ void k_row_count(uint32_t n, const uint32_t* __restrict__ ptr, const 
 
 __global__ void k_scatter_core(uint32_t n, const uint32_t* __restrict__ ptr, const uint8_t* __restrict__ flags,
                                const uint32_t* __restrict__ cptr, const uint32_t* __restrict__ adj,
-                               const uint2* __restrict__ adjw, uint32_t* __restrict__ cadj, uint2* __restrict__ cadjw) {
+                               const uint2* __restrict__ adjw, uint32_t* __restrict__ cadj, uint2* __restrict__ cadjw,
+                               int inv = 0) {
     const uint32_t lane = threadIdx.x & 31;
     const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
     for (uint64_t u = blockIdx.x * (uint64_t)(blockDim.x / 32) + (threadIdx.x >> 5); u < n; u += nw) {
@@ -172,7 +174,7 @@ __global__ void k_scatter_core(uint32_t n, const uint32_t* __restrict__ ptr, con
         const uint32_t r0 = ptr[u], r1 = ptr[u + 1];
         for (uint32_t b = r0; b < r1; b += 32) {
             const uint32_t e = b + lane;
-            const bool f = e < r1 && flags[e];
+            const bool f = e < r1 && ((flags[e] != 0) != (inv != 0));
             const uint32_t bal = __ballot_sync(FULLM, f);
             if (f) {
                 const uint32_t p = o + __popc(bal & ((1u << lane) - 1u));
@@ -427,7 +429,20 @@ void finalize_core(Graph& G, int kind, Core& C, int connectivity, cudaStream_t s
     C.adj.adjw.reset();
     if (G.packed) C.adj.adj.alloc(adj_alloc_elems(mcg, 4), s); else C.adj.adjw.alloc(adj_alloc_elems(mcg, 8), s);
     CGB_LAUNCH(k_scatter_core, grid_rows(G.n), TB, 0, s, G.n, G.g.ptr.get(), C.flags.get(), C.adj.ptr.get(),
-               G.g.adj.get(), G.g.adjw.get(), C.adj.adj.get(), C.adj.adjw.get());
+               G.g.adj.get(), G.g.adjw.get(), C.adj.adj.get(), C.adj.adjw.get(), 0);
+    // G minus the CG (reading N7, the split-CSR benefit P:2567-2572): after phase 1 every CG
+    // edge is at its fixpoint, so phase 2's first sweep relaxes only these edges
+    C.rest.n = G.n;
+    C.rest.ptr.alloc(G.n + 1, s);
+    CGB_LAUNCH(k_row_count, grid_rows(G.n + 1), TB, 0, s, G.n, G.g.ptr.get(), C.flags.get(), cnt.get(), 1);
+    exclusive_sum(cnt.get(), C.rest.ptr.get(), (uint64_t)G.n + 1, s);
+    C.rest.m = G.m - mcg;
+    C.rest.adj.reset();
+    C.rest.adjw.reset();
+    if (G.packed) C.rest.adj.alloc(adj_alloc_elems(C.rest.m, 4), s); else C.rest.adjw.alloc(adj_alloc_elems(C.rest.m, 8), s);
+    CGB_LAUNCH(k_scatter_core, grid_rows(G.n), TB, 0, s, G.n, G.g.ptr.get(), C.flags.get(), C.rest.ptr.get(),
+               G.g.adj.get(), G.g.adjw.get(), C.rest.adj.get(), C.rest.adjw.get(), 1);
+    C.rest_built = true;
 }
 
 struct Timer {

@@ -68,6 +68,8 @@ struct BParams {
     uint32_t max_iters;
     uint32_t bits_below;        // frontiers smaller than this keep a bitmap (else the masks M are scanned)
     GraphView R;                // G^R: in-edges for the NEXT-1 pull
+    GraphView Rst;              // G minus the CG: phase 2's first sweep (reading N7)
+    int use_rest;
     const uint32_t* HB;         // CG hub rows [n][2K] for the certificates (nullable; u32 lanes only)
     uint32_t K, KP;             // hubs in HB; row stride 2*KP (KP = K rounded up to a multiple of 4)
     int reduced;                // phase 2 starts with the certificate-driven pull (NEXT-1)
@@ -1122,7 +1124,9 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
         bool pull = false;       // this iteration is the NEXT-1 pull over uncertified vertices
         uint32_t iters = 0, n_edges = 0, n_upd = 0, n_read = 0;  // (edge, query) pairs / edge reads
         for (;;) {
-            const GraphView& g = (phase == 1) ? P.C : P.G;
+            // phase 2's first sweep (Alg 3 l.15 seeding, `predicate`) relaxes G minus the CG:
+            // every CG edge is at its fixpoint after phase 1 (reading N7)
+            const GraphView& g = (phase == 1) ? P.C : (predicate && P.use_rest) ? P.Rst : P.G;
             const bool fresh = (P.fresh >> (phase - 1)) & 1u;
             const int slot = ring & 3;
             unsigned long long* ctr = P.ctrl + CT0 + CTS * slot;
@@ -1336,6 +1340,9 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
         const bool hub_cert = lw == 32 && core.hub_k > 0 && core.hub_k <= 64 && core.hub_vals.get();
         const bool has_cert = c.kind == CG_REACH || hub_cert;
         P.reduced = c.two_phase && c.core_adj == &core.adj && ((mask >> c.kind) & 1u) && has_cert;
+        const char* rs = getenv("CG_REST");
+        P.use_rest = c.two_phase && c.core_adj == &core.adj && core.rest_built && (rs ? atoi(rs) : 1);
+        if (P.use_rest) P.Rst = view(core.rest);
         if (P.reduced && c.kind != CG_REACH) {
             P.HB = core.hub_vals.get();
             P.K = core.hub_k;

@@ -43,6 +43,8 @@ struct Core {
     // queries' values kept as rows hub_vals[v][0..2K) = (Q(h_k) on G at v | Q(h_k) on G^R at v)
     DevBuf<uint32_t> hub_vals;
     uint32_t hub_k = 0;
+    Adj rest;              // G minus the CG (phase 2's first sweep, reading N7)
+    bool rest_built = false;
     Adj sym;               // WCC: CG ∪ CG^R (built on the first WCC 2Phase query)
     bool sym_built = false;
 };

@@ -306,6 +306,32 @@ def test_single_and_batched_engines(engine, monkeypatch):
                 (ost["reached"], ost["precise_p1"], ost["impacted"]), (batch, kind, int(s))
 
 
+@pytest.mark.parametrize("rest", ["0", "1"])
+def test_first_sweep_over_g_minus_cg(rest, monkeypatch):
+    """Reading N7: after phase 1 every CG edge is at its fixpoint, so phase 2's first sweep may
+    relax only G minus the CG (CG_REST=1, the default) — values, phase-1 values and the
+    reached / precise / impacted counts are those of the full first sweep (CG_REST=0) and the
+    oracle's, for every kind, with an Alg 1 CG (connectivity edges included) and Alg 2's."""
+    monkeypatch.setenv("CG_REST", rest)
+    n, m = 1 << 15, 16 << 15
+    src, dst, w = gen.rmat(n, m, w_max=17, seed=41)
+    g, og = both(n, src, dst, w)
+    ogr = oracle.transpose(og)
+    hubs = oracle.hubs_topdeg(og, ogr, 20)
+    sources = np.concatenate([[0], gen.sample_sources(n, src, dst, 36, seed=5)]).astype(np.uint32)
+    for kind in KINDS:
+        g.build(kind, K=20)
+        cg = oracle.subgraph(og, oracle.cg_for_kind(kind, og, ogr, hubs))
+        out, p1, st = g.query(kind, to_dev(sources), mode="2phase", p1=True, stats=True)
+        out, p1 = to_np(out), to_np(p1)
+        for i, s in enumerate(sources):
+            val, op1, ost = oracle.two_phase(kind, og, cg, int(s))
+            assert_values_equal(out[i], val, kind, f"rest={rest} {kind} s={s}")
+            assert_values_equal(p1[i], op1, kind, f"rest={rest} {kind} p1 s={s}")
+            assert (st[i]["reached"], st[i]["precise_p1"], st[i]["impacted"]) == \
+                (ost["reached"], ost["precise_p1"], ost["impacted"]), (rest, kind, int(s))
+
+
 @pytest.mark.parametrize("bits_below", ["0", "4294967295"])
 def test_batched_frontier_modes(bits_below, monkeypatch):
     """The batched engine keeps the union frontier either as bitmap bits set by S2 or as the
