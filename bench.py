@@ -423,7 +423,10 @@ def main():
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                 "traffic": traffic, "kernel": "batch_kernel<KIND,packed,lanes> (one launch per kind per step)",
                 "peak_source": peak_src,
-                "alg_bytes_per_launch": tot_bytes / len(kinds)}
+                "alg_bytes_per_launch": tot_bytes / len(kinds),
+                "achieved_how": "algorithmic bytes (cg_stats counters, DESIGN.md §7) summed over the kinds' "
+                                "launches / their summed CUDA-event durations on the launching stream",
+                "traffic_how": (tr["how"] + " (" + tr["report"] + ")") if tr else None}
 
     # ---- NEXT-3 WCC (a whole-graph query, reported beside the six-kind headline): 2Phase on
     # REACH's general CG vs FULL, device-timed, same warm-up rule
