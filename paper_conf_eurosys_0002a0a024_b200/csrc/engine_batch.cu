@@ -45,7 +45,7 @@ constexpr int S_PIPE = CGB_STAGES;  // value-row pipeline depth (chunks of 32 ed
 constexpr int E_AHEAD = CGB_EAHEAD;  // edge-word lead over the row requests (chunks)
 
 enum { ST_IT1, ST_IT2, ST_E1, ST_E2, ST_U1, ST_U2, ST_F1, ST_F2, ST_IMP, ST_REACH, ST_PREC, ST_S1, ST_S2, NSTAT };
-enum { CT0 = 8, CTS = 2, CT_LIST = 0, CT_ACTIVE = 1 };
+enum { CT0 = 8, CTS = 3, CT_LIST = 0, CT_ACTIVE = 1, CT_TILE = 2 };
 enum { ERR_ITERS = 1u, ERR_SOURCE = 2u, ERR_LANE_OVERFLOW = 4u };
 
 struct BParams {
@@ -70,12 +70,14 @@ struct BParams {
     GraphView R;                // G^R: in-edges for the NEXT-1 pull
     GraphView Rst;              // G minus the CG: phase 2's first sweep (reading N7)
     int use_rest;
+    int dyn;                    // S2's second half in dynamically taken tiles
     const uint32_t* HB;         // CG hub rows [n][2K] for the certificates (nullable; u32 lanes only)
     uint32_t K, KP;             // hubs in HB; row stride 2*KP (KP = K rounded up to a multiple of 4)
     int reduced;                // phase 2 starts with the certificate-driven pull (NEXT-1)
     uint32_t fresh;             // bit p-1: phase p pre-reads values from L2 instead of L1
     unsigned long long* trace;  // nullable: per iteration {t_start, t_s1, t_s2, phase<<62|q0<<32|listed, active<<32|edges}
     uint32_t trace_cap;
+    unsigned long long* trace_cta;  // nullable: per iteration {first, last} CTA S2 finish times
 };
 
 // ------------------------------------------------------------------ value lanes
@@ -796,14 +798,12 @@ constexpr bool xs_double() { return L::RW <= 16; }
 // are prefetched one ahead: while window i's edges run, window i+1's source rows are already
 // being copied (cp.async) into the other half of xs and window i+2's list entries are loading.
 template <int KIND, bool PACKED, class L>
-__device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, uint32_t E, uint32_t* xs, uint32_t* vs,
-                        bool set_bits, bool fresh, uint32_t& n_edges, uint32_t& n_upd, uint32_t& n_read) {
+__device__ void relax_range(const BParams& P, const GraphView& g, uint32_t count, uint32_t E, uint32_t e0, uint32_t e1,
+                            uint32_t* xs, uint32_t* vs, bool set_bits, bool fresh, uint32_t& n_edges, uint32_t& n_upd,
+                            uint32_t& n_read) {
     constexpr int RW = L::RW;
     using RC = RowCopy<L>;
     const uint32_t lane = threadIdx.x & 31;
-    const uint32_t gw = blockIdx.x * BW + (threadIdx.x >> 5);
-    const uint64_t NW = (uint64_t)gridDim.x * BW;
-    const uint32_t e0 = (uint32_t)((uint64_t)E * gw / NW), e1 = (uint32_t)((uint64_t)E * (gw + 1) / NW);
     if (e0 >= e1) return;
     auto list_load = [&](uint32_t i0, uint32_t& v, uint32_t& off, uint32_t& mask) {
         const uint32_t idx = i0 + lane;
@@ -861,6 +861,37 @@ __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, ui
         nv = mv;
         noff = moff;
         nmask = mmask;
+    }
+}
+
+// The iteration's E list edges over all warps: a static half split evenly (edge-balanced), then
+// — for iterations long enough to amortise a tile's list search — the rest in tiles taken from
+// a per-iteration counter, so warps slowed by contended EdgeFunctions (phase 1's hub rows) do
+// not hold the grid barrier (trace: the last CTA finished 33 % after the first without it).
+#ifndef CGB_DYN_MIN
+#define CGB_DYN_MIN 1024u  // edges per warp below which the split stays fully static (measured 512 / 1024 / 2048)
+#endif
+template <int KIND, bool PACKED, class L>
+__device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, uint32_t E, uint32_t* xs, uint32_t* vs,
+                        bool set_bits, bool fresh, uint32_t& n_edges, uint32_t& n_upd, uint32_t& n_read,
+                        unsigned long long* tiles) {
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t gw = blockIdx.x * BW + (threadIdx.x >> 5);
+    const uint64_t NW = (uint64_t)gridDim.x * BW;
+    const bool dyn = tiles != nullptr && (uint64_t)E >= NW * CGB_DYN_MIN;
+    const uint32_t Es = dyn ? E / 2 : E;
+    const uint32_t T = dyn ? max(1024u, (uint32_t)((E - Es + NW - 1) / NW)) : 0u;
+    uint32_t a = (uint32_t)((uint64_t)Es * gw / NW), b = (uint32_t)((uint64_t)Es * (gw + 1) / NW);
+    for (;;) {  // one call site: the range body is inlined once
+        relax_range<KIND, PACKED, L>(P, g, count, E, a, b, xs, vs, set_bits, fresh, n_edges, n_upd, n_read);
+        if (!dyn) break;
+        unsigned long long t = 0;
+        if (lane == 0) t = atomicAdd(tiles, 1ull);
+        t = __shfl_sync(FULL, t, 0);
+        const uint64_t a64 = Es + t * T;
+        if (a64 >= E) break;
+        a = (uint32_t)a64;
+        b = (uint32_t)(a64 + T < E ? a64 + T : E);
     }
 }
 
@@ -1132,7 +1163,7 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
             unsigned long long* ctr = P.ctrl + CT0 + CTS * slot;
             if (tid == 0) {
                 unsigned long long* z = P.ctrl + CT0 + CTS * ((ring + 2) & 3);
-                z[0] = z[1] = 0ull;
+                z[0] = z[1] = z[2] = 0ull;
             }
             const unsigned long long t_s0 = (P.trace && tid == 0) ? global_ns() : 0ull;
             const int mode = pull ? F_UNCERT : predicate ? F_IMPACTED : bits ? F_BITS : F_MASKS;
@@ -1205,8 +1236,17 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
                 // small frontier: its S2 sets frontier bits (few reds) and the next S1 reads the
                 // bitmap; large frontier: no bitmap reds (they contend in L2), the next S1 scans M
                 bits = E < P.bits_below;  // at most E vertices change
-                relax_b<KIND, PACKED, L>(P, g, count, E, xs, vs, bits, fresh, n_edges, n_upd, n_read);
+                relax_b<KIND, PACKED, L>(P, g, count, E, xs, vs, bits, fresh, n_edges, n_upd, n_read,
+                                         P.dyn ? ctr + CT_TILE : nullptr);
                 predicate = false;
+            }
+            if (P.trace_cta && tr + 1 < P.trace_cap) {  // S2 load balance across CTAs (trace only)
+                __syncthreads();
+                if (threadIdx.x == 0) {
+                    const unsigned long long tn = global_ns();
+                    atomicMin(P.trace_cta + 2ull * tr, tn);
+                    atomicMax(P.trace_cta + 2ull * tr + 1, tn);
+                }
             }
             grid_sync(P.ctrl, epoch);
             if (P.trace && tid == 0 && tr + 1 < P.trace_cap) P.trace[5ull * tr + 2] = global_ns();
@@ -1340,6 +1380,8 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
         const bool hub_cert = lw == 32 && core.hub_k > 0 && core.hub_k <= 64 && core.hub_vals.get();
         const bool has_cert = c.kind == CG_REACH || hub_cert;
         P.reduced = c.two_phase && c.core_adj == &core.adj && ((mask >> c.kind) & 1u) && has_cert;
+        const char* dy = getenv("CG_DYN");
+        P.dyn = dy ? atoi(dy) : 1;
         const char* rs = getenv("CG_REST");
         P.use_rest = c.two_phase && c.core_adj == &core.adj && core.rest_built && (rs ? atoi(rs) : 1);
         if (P.use_rest) P.Rst = view(core.rest);
@@ -1375,19 +1417,27 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
     CGB_CUDA(cudaMemsetAsync(w.err.get(), 0, 4, s));
     if (stats) CGB_CUDA(cudaMemsetAsync(st.get(), 0, st.bytes(), s));
     static const bool tracing = getenv("CG_TRACE") != nullptr;
-    DevBuf<unsigned long long> trace;
+    DevBuf<unsigned long long> trace, trace_cta;
+    P.trace_cta = nullptr;
     if (tracing) {
         P.trace_cap = 1u << 16;
         trace.alloc(5ull * P.trace_cap, s);
         CGB_CUDA(cudaMemsetAsync(trace.get(), 0, trace.bytes(), s));
         P.trace = trace.get();
+        trace_cta.alloc(2ull * P.trace_cap, s);
+        std::vector<unsigned long long> init(2ull * P.trace_cap);
+        for (size_t i = 0; i < init.size(); i += 2) init[i] = ~0ull, init[i + 1] = 0ull;
+        CGB_CUDA(cudaMemcpyAsync(trace_cta.get(), init.data(), trace_cta.bytes(), cudaMemcpyHostToDevice, s));
+        CGB_CUDA(cudaStreamSynchronize(s));
+        P.trace_cta = trace_cta.get();
     }
     if (G.packed) launch_kind_b<true>(c.kind, lw, P, G.num_sms, s);
     else launch_kind_b<false>(c.kind, lw, P, G.num_sms, s);
     CGB_CUDA(cudaMemcpyAsync(err_out, w.err.get(), 4, cudaMemcpyDeviceToHost, s));
     if (tracing) {
-        std::vector<unsigned long long> h(5ull * P.trace_cap);
+        std::vector<unsigned long long> h(5ull * P.trace_cap), hc(2ull * P.trace_cap);
         CGB_CUDA(cudaMemcpyAsync(h.data(), trace.get(), trace.bytes(), cudaMemcpyDeviceToHost, s));
+        CGB_CUDA(cudaMemcpyAsync(hc.data(), trace_cta.get(), trace_cta.bytes(), cudaMemcpyDeviceToHost, s));
         CGB_CUDA(cudaStreamSynchronize(s));
         unsigned long long t0 = 0;
         {
@@ -1399,9 +1449,11 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
             const unsigned long long* t = h.data() + 5 * i;
             if (!t0) t0 = t[0];
             fprintf(stderr, "CG_TRACE kind=%d Q=%d lanes=%d it=%u q0=%llu phase=%llu list=%llu active=%llu edges=%llu "
-                    "t=%.1f s1=%.1f s2=%.1f us\n", c.kind, Q, lw, i, (t[3] >> 32) & 0x3fffffffull, t[3] >> 62,
-                    t[3] & 0xffffffffull, t[4] >> 32, t[4] & 0xffffffffull, (t[0] - t0) / 1e3, (t[1] - t[0]) / 1e3,
-                    t[2] ? (t[2] - t[1]) / 1e3 : 0.0);
+                    "t=%.1f s1=%.1f s2=%.1f us s2_cta_first=%.1f s2_cta_last=%.1f\n", c.kind, Q, lw, i,
+                    (t[3] >> 32) & 0x3fffffffull, t[3] >> 62, t[3] & 0xffffffffull, t[4] >> 32, t[4] & 0xffffffffull,
+                    (t[0] - t0) / 1e3, (t[1] - t[0]) / 1e3, t[2] ? (t[2] - t[1]) / 1e3 : 0.0,
+                    hc[2 * i + 1] ? ((double)hc[2 * i] - (double)t[1]) / 1e3 : 0.0,
+                    hc[2 * i + 1] ? ((double)hc[2 * i + 1] - (double)t[1]) / 1e3 : 0.0);
         }
     }
     if (stats) {
