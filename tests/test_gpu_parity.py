@@ -332,6 +332,24 @@ def test_first_sweep_over_g_minus_cg(rest, monkeypatch):
                 (ost["reached"], ost["precise_p1"], ost["impacted"]), (rest, kind, int(s))
 
 
+@pytest.mark.parametrize("dyn", ["0", "1"])
+def test_static_and_dynamic_s2_split(dyn, monkeypatch):
+    """S2's edge split: fully static (CG_DYN=0) or half static + tiles taken from a per-iteration
+    counter (the default for iterations with >= 1,024 list edges per warp, i.e. >= 2.4 M edges:
+    the dense iterations of RMAT-18 with 32 sources)."""
+    monkeypatch.setenv("CG_DYN", dyn)
+    n, m = 1 << 18, 16 << 18
+    src, dst, w = gen.rmat(n, m, w_max=19, seed=17)
+    g, og = both(n, src, dst, w)
+    sources = gen.sample_sources(n, src, dst, 32, seed=12)
+    for kind in ("sssp", "viterbi", "bfs"):
+        g.build(kind, K=20)
+        for mode in ("2phase", "full"):
+            out = to_np(g.query(kind, to_dev(sources), mode=mode))
+            for i, s in enumerate(sources[:8]):
+                assert_values_equal(out[i], oracle.query(kind, og, int(s)), kind, f"dyn={dyn} {kind} {mode}")
+
+
 @pytest.mark.parametrize("bits_below", ["0", "4294967295"])
 def test_batched_frontier_modes(bits_below, monkeypatch):
     """The batched engine keeps the union frontier either as bitmap bits set by S2 or as the
