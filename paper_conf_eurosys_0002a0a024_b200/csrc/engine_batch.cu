@@ -642,7 +642,10 @@ __device__ __forceinline__ void window_edges(const BParams& P, const GraphView& 
                                              uint32_t off, uint32_t base, uint32_t mask, uint32_t e, uint32_t ehi,
                                              bool set_bits, bool fresh, uint32_t& n_edges, uint32_t& n_upd,
                                              uint32_t& n_read) {
-    constexpr int S = S_PIPE, EA = E_AHEAD, RW = L::RW;
+    // binary16 rows (the cheapest relax per edge) keep the edge stream 4 chunks ahead; the u32
+    // rows' heavier relax needs the registers (measured: Viterbi 16 % slower with 4)
+    constexpr int EA = (L::QPW == 2 && E_AHEAD == S_PIPE) ? 2 * S_PIPE : E_AHEAD;
+    constexpr int S = S_PIPE, RW = L::RW;
     static_assert(EA % S == 0 && EA >= S, "E_AHEAD must be a multiple of S_PIPE");
     using RC = RowCopy<L>;
     constexpr uint32_t NONE = 0xffffffffu;
