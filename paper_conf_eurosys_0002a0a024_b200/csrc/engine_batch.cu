@@ -91,9 +91,12 @@ struct BParams {
 //   relax(p, uw, cw, w, act, ...)  Process + EdgeFunction of one word (Alg 3 l.22-27): the lanes
 //       of act whose candidate ext(uw, w) is better than cw; returns the changed lanes
 template <int KIND, int QN>
-struct Lanes32 {  // one u32 per query (Table 6 types), QN queries per pass, 4 words (16 B) per relax group
+struct Lanes32 {  // one u32 per query (Table 6 types), QN queries per pass, CGB_G32 words per relax group
     using O = Op<KIND>;
-    static constexpr int Q = QN, QPW = 1, RW = QN, G = 4;
+#ifndef CGB_G32
+#define CGB_G32 16  // queries per relax group (measured on C2 Viterbi: 4 -> 5.06 ms, 8 -> 4.76, 16 -> 4.65)
+#endif
+    static constexpr int Q = QN, QPW = 1, RW = QN, G = CGB_G32;
     __device__ static uint32_t init_word() { return O::INIT; }
     __device__ static uint32_t decode(uint32_t x, uint32_t) { return x; }
     __device__ static uint32_t live(uint32_t x) { return x != O::INIT; }
@@ -107,7 +110,7 @@ struct Lanes32 {  // one u32 per query (Table 6 types), QN queries per pass, 4 w
         if constexpr (VIT) return vit_arg(w);
         else return w;
     }
-    // Process + EdgeFunction of 4 queries: candidates and Needed tests for all 4 without
+    // Process + EdgeFunction of G queries: candidates and Needed tests for all G without
     // branches, then one EdgeFunction per needed query (act: 4 query bits; an unreached u —
     // a pull may read one — is never Needed).
     __device__ static uint32_t relax(uint32_t* p, const uint32_t (&u)[G], const uint32_t (&c)[G], const Arg& w,

@@ -62,13 +62,14 @@ __device__ __forceinline__ uint32_t vit_div(uint32_t a, const VitArg& A) {
     return __float_as_uint(y);
 }
 
-// four quotients of one edge (a batch row's 16 B group): the fast path for all four, one
+// the N quotients of one edge (a batch row's relax group): the fast path for all N, one
 // warp-divergent branch to __fdiv_rn only when some lane falls outside it
-__device__ __forceinline__ void vit_div4(const uint32_t (&a)[4], const VitArg& A, uint32_t (&out)[4]) {
+template <int N>
+__device__ __forceinline__ void vit_div4(const uint32_t (&a)[N], const VitArg& A, uint32_t (&out)[N]) {
     const float b = __uint2float_rn(A.w);
     bool slow = A.r == 0.0f;
 #pragma unroll
-    for (int i = 0; i < 4; ++i) {
+    for (int i = 0; i < N; ++i) {
         const float x = __uint_as_float(a[i]);
         const float q = __fmul_rn(x, A.r);
         const float e = __fmaf_rn(-q, b, x);
@@ -77,7 +78,7 @@ __device__ __forceinline__ void vit_div4(const uint32_t (&a)[4], const VitArg& A
     }
     if (slow) {
 #pragma unroll
-        for (int i = 0; i < 4; ++i) out[i] = vit_div(a[i], A);
+        for (int i = 0; i < N; ++i) out[i] = vit_div(a[i], A);
     }
 }
 
