@@ -149,7 +149,10 @@ struct Lanes32 {  // one u32 per query (Table 6 types), QN queries per pass, CGB
 template <int KIND>
 struct Lanes16 {
     static_assert(KIND == CG_SSSP || KIND == CG_SSWP || KIND == CG_SSNP || KIND == CG_BFS, "f16 lanes");
-    static constexpr int Q = 32, QPW = 2, RW = 16, G = 4;
+#ifndef CGB_G16
+#define CGB_G16 16  // measured on C2: 4 -> 11.54 K q/s, 8 -> 11.83 K, 16 -> 11.89 K
+#endif
+    static constexpr int Q = 32, QPW = 2, RW = 16, G = CGB_G16;  // words per relax group (multiple of 4)
     using Arg = uint32_t;
     __device__ static Arg arg(uint32_t w) { return w; }
     static constexpr bool MAXK = KIND == CG_SSWP;
@@ -214,14 +217,18 @@ struct Lanes16 {
             ch |= bits2(bm[i]) << (2 * i);
         }
         if (over) atomicOr(err, ERR_LANE_OVERFLOW);
-        if (MAXK)
-            asm volatile("red.relaxed.gpu.global.max.noftz.v4.f16x2 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(x[0]),
-                         "r"(x[1]), "r"(x[2]), "r"(x[3])
-                         : "memory");
-        else
-            asm volatile("red.relaxed.gpu.global.min.noftz.v4.f16x2 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(x[0]),
-                         "r"(x[1]), "r"(x[2]), "r"(x[3])
-                         : "memory");
+#pragma unroll
+        for (int h = 0; h < G / 4; ++h) {  // one 16 B vector EdgeFunction per 8 queries with a needed lane
+            if (!((ch >> (8 * h)) & 0xffu)) continue;
+            if (MAXK)
+                asm volatile("red.relaxed.gpu.global.max.noftz.v4.f16x2 [%0], {%1,%2,%3,%4};" ::"l"(p + 4 * h),
+                             "r"(x[4 * h]), "r"(x[4 * h + 1]), "r"(x[4 * h + 2]), "r"(x[4 * h + 3])
+                             : "memory");
+            else
+                asm volatile("red.relaxed.gpu.global.min.noftz.v4.f16x2 [%0], {%1,%2,%3,%4};" ::"l"(p + 4 * h),
+                             "r"(x[4 * h]), "r"(x[4 * h + 1]), "r"(x[4 * h + 2]), "r"(x[4 * h + 3])
+                             : "memory");
+        }
         n_upd += __popc(ch);
         return ch;
     }
