@@ -18,6 +18,18 @@
  *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default
  *     stream).  cg_query / cg_rmat_generate are stream-ordered and
  *     asynchronous; cg_graph_create and cg_build synchronise `stream`.
+ *   - All calls on one cg_graph share its device workspace.  They may be
+ *     issued on different streams: each call's stream first waits (an event,
+ *     no host sync) for the previous call on that graph, so the calls run in
+ *     issue order.  Calls on one graph must come from one host thread at a
+ *     time.
+ *   - Errors detected on the DEVICE by an asynchronous call (a source id >= n
+ *     in a device array, a narrow output format overflow, an internal
+ *     iteration bound) are STICKY per graph: the next query call on the graph
+ *     (cg_query*, cg_query_host*) returns that error without doing its own
+ *     work, and cg_graph_status() synchronises `stream` and returns it.  Either
+ *     clears it.  Calls with `stats` synchronise and return their own device
+ *     errors directly.
  *   - No PyTorch types appear here; the Python binding passes raw pointers
  *     (torch tensors' data_ptr) and a raw stream handle.
  *   - Internal device memory comes from the allocator installed with
@@ -40,7 +52,8 @@ typedef enum {
     CG_ENOMEM = -2,        /* device allocation failed */
     CG_ECUDA = -3,         /* a CUDA runtime error (detail in cg_last_error) */
     CG_ENOCG = -4,         /* cg_query(..., CG_MODE_2PHASE) before cg_build for that kind */
-    CG_EOVERFLOW = -5,     /* n >= 2^32-1, m >= 2^32, or (n-1)*w_max >= 2^32-1 (SSSP could wrap) */
+    CG_EOVERFLOW = -5,     /* n >= 2^32-1, m >= 2^32, or (n-1)*w_max >= 2^32-1 (SSSP could wrap);
+                              a value not representable in the requested narrow output format */
     CG_EUNSUPPORTED = -7,  /* feature not available on this device (e.g. no cooperative launch) */
     CG_EINTERNAL = -8      /* internal invariant violated (e.g. iteration bound exceeded) */
 } cg_status;
@@ -56,6 +69,15 @@ typedef enum { CG_SSSP = 0, CG_SSWP = 1, CG_SSNP = 2, CG_VITERBI = 3, CG_BFS = 4
  * query: cg_query takes n_src == 1 (src may be NULL) and writes n labels.  2PHASE runs phase 1
  * on the general Core Graph (Alg 2, shared with BFS / REACH) and phase 2 on G from every
  * vertex (reading W2). */
+
+/* Output formats of the value rows (cg_query_fmt / cg_query_host_fmt).  The values are the same;
+ * only their encoding differs (a narrower wire format for gathers and host copies):
+ *   CG_OUT_U32   row q = n uint32 words (binary32 for VITERBI) — cg_query's format;
+ *   CG_OUT_U16   row q = n uint16: a value < 0xFFFF as itself, 0xFFFFFFFF (InitVal of SSSP / SSNP /
+ *                BFS, SourceInitVal of SSWP) as 0xFFFF; any other value >= 0xFFFF is a sticky
+ *                CG_EOVERFLOW.  SSSP, SSWP, SSNP, BFS, REACH (not VITERBI, not WCC);
+ *   CG_OUT_BITS  REACH only: row q = ceil(n/32) uint32 words, bit (v % 32) of word v/32 = Val(v). */
+typedef enum { CG_OUT_U32 = 0, CG_OUT_U16 = 1, CG_OUT_BITS = 2 } cg_out_format;
 
 /* CG_MODE_2PHASE: Algorithm 3 — phase 1 on the Core Graph, phase 2 on G
  * from the impacted set.  CG_MODE_FULL: the baseline, the same relaxation on G only. */
@@ -74,7 +96,7 @@ typedef enum { CG_ALG_AUTO = 0, CG_ALG_SPECIALIZED = 1, CG_ALG_GENERAL = 2, CG_A
 
 typedef struct cg_graph_s* cg_graph; /* opaque: owns G (CSR), G^R (CSC) and the CGs on one device */
 
-/* Per-query counters (SURVEY §5 tracing; Table 5 / Fig 5 analogs).  Edge and update
+/* Per-query counters (SURVEY §5 tracing; Table 5 / Fig 5 analogs; SURVEY §8(b) cg_stats).  Edge and update
  * counts of the asynchronous GPU relaxation are NOT unique (they depend on timing);
  * impacted / reached / precise_p1 ARE unique.  When queries run batched (several sources per
  * pass, the default for n_src >= 2), iterations and frontier sizes are those of the batch's
@@ -94,7 +116,11 @@ typedef struct {
                                         read once for all queries of the batch, split evenly over them */
     int32_t batch_queries;           /* queries per pass of the engine that ran this query (1: single-query) */
     int32_t row_bytes;               /* bytes of one vertex's value row in that pass (u32 lanes: 4 per query;
-                                        u8 lanes: 1 per query; REACH bit lanes: 1 bit per query) */
+                                        binary16 lanes: 2 per query; REACH bit lanes: 1 bit per query) */
+    float ms_p1;                     /* device time of init + phase 1 (Alg 3 l.3-13) of the pass that ran
+                                        this query (0 in FULL mode: everything is phase 2) */
+    float ms_p2;                     /* device time of phase 2 (l.14-18) + writing the values out; the
+                                        queries of one batched pass share their pass's two times */
 } cg_stats;
 
 typedef void* (*cg_alloc_fn)(size_t bytes, void* stream, void* ctx);
@@ -185,13 +211,26 @@ cg_status cg_core_export(cg_graph g, cg_kind kind, uint8_t* flags, void* stream)
  * CG_MODE_FULL.  The results of both modes are identical.
  * p1_out (device, nullable): phase-1 values per query (2PHASE only), enables precise_p1.
  * stats (host, nullable, n_src entries): per-query counters; if non-NULL the call
- * synchronises `stream`, else it is fully asynchronous (one persistent kernel launch).
- * Errors: CG_EINVAL, CG_ENOCG, CG_ENOMEM, CG_ECUDA, CG_EINTERNAL.
+ * synchronises `stream` and reports this call's device errors; else it is fully asynchronous
+ * (no host synchronisation; one persistent kernel launch, plus for SSSP / BFS a second launch
+ * that exits at once unless the binary16 value lanes overflowed, reading N3) and device errors
+ * are sticky (see the conventions above).
+ * Errors: CG_EINVAL (also: n_src > 0 with a NULL src, except CG_WCC), CG_ENOCG, CG_ENOMEM,
+ * CG_ECUDA, CG_EINTERNAL, or a pending sticky error of an earlier call.
  */
 cg_status cg_query(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode, void* out,
                    cg_stats* stats, void* stream);
 cg_status cg_query_ex(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode, void* out,
                       void* p1_out, cg_stats* stats, void* stream);
+
+/* cg_query_ex with an output format (cg_out_format): out holds n_src rows in that format. */
+cg_status cg_query_fmt(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode,
+                       cg_out_format fmt, void* out, void* p1_out, cg_stats* stats, void* stream);
+
+/* Synchronise `stream`, then return (and clear) the graph's sticky device error (CG_OK if none):
+ * CG_EINVAL for a source id >= n passed in a device array to an asynchronous query (its row holds
+ * InitVal), CG_EOVERFLOW for a narrow-format overflow, CG_EINTERNAL for an iteration bound. */
+cg_status cg_graph_status(cg_graph g, void* stream);
 
 /*
  * End-to-end variant with HOST buffers: src (host, n_src ids) and out (host, n_src*n words).
@@ -201,6 +240,9 @@ cg_status cg_query_ex(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_s
  */
 cg_status cg_query_host(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode, void* out,
                         int32_t batch, void* stream);
+/* The same with an output format (cg_out_format): out (host) holds n_src rows in that format. */
+cg_status cg_query_host_fmt(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode,
+                            cg_out_format fmt, void* out, int32_t batch, void* stream);
 
 /*
  * Device twin of the seeded R-MAT input generator (gen/rmat.c defines it): edges

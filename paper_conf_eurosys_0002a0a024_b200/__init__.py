@@ -6,8 +6,8 @@ The CUDA library (csrc/ -> libcoregraph_b200.so) is the only compute path; there
 fallback.  ``Graph`` marshals tensors to the ABI.
 """
 from . import multi  # noqa: F401
-from .graph import CG_ALGS, HUB_POLICIES, KINDS, MODES, Graph, kernel_launches, kind_id, rmat_device  # noqa: F401
+from .graph import CG_ALGS, FORMATS, HUB_POLICIES, KINDS, MODES, Graph, kernel_launches, kind_id, rmat_device  # noqa: F401
 from ._lib import CGError, CGInvalid, CGNoCoreGraph, CGOverflow, CGUnsupported  # noqa: F401
 
-__all__ = ["Graph", "rmat_device", "KINDS", "MODES", "HUB_POLICIES", "CG_ALGS", "kernel_launches", "kind_id",
+__all__ = ["Graph", "rmat_device", "KINDS", "MODES", "FORMATS", "HUB_POLICIES", "CG_ALGS", "kernel_launches", "kind_id",
            "CGError", "CGInvalid", "CGNoCoreGraph", "CGOverflow", "CGUnsupported"]

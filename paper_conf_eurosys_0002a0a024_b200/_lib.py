@@ -54,10 +54,12 @@ class Stats(ctypes.Structure):
                 ("impacted", ctypes.c_int64), ("reached", ctypes.c_int64),
                 ("precise_p1", ctypes.c_int64),
                 ("scanned_p1", ctypes.c_int64), ("scanned_p2", ctypes.c_int64),
-                ("batch_queries", ctypes.c_int32), ("row_bytes", ctypes.c_int32)]
+                ("batch_queries", ctypes.c_int32), ("row_bytes", ctypes.c_int32),
+                ("ms_p1", ctypes.c_float), ("ms_p2", ctypes.c_float)]
 
     def as_dict(self) -> dict:
-        return {k: int(getattr(self, k)) for k, _ in self._fields_}
+        return {k: (float(getattr(self, k)) if k.startswith("ms_") else int(getattr(self, k)))
+                for k, _ in self._fields_}
 
 
 ALLOC_FN = ctypes.CFUNCTYPE(ctypes.c_void_p, ctypes.c_size_t, ctypes.c_void_p, ctypes.c_void_p)
@@ -86,7 +88,12 @@ _SIGS = {
     "cg_core_load": (ctypes.c_int, [_P, ctypes.c_int, ctypes.c_char_p, _P]),
     "cg_query": (ctypes.c_int, [_P, ctypes.c_int, _P, ctypes.c_int32, ctypes.c_int, _P, _P, _P]),
     "cg_query_ex": (ctypes.c_int, [_P, ctypes.c_int, _P, ctypes.c_int32, ctypes.c_int, _P, _P, _P, _P]),
+    "cg_query_fmt": (ctypes.c_int, [_P, ctypes.c_int, _P, ctypes.c_int32, ctypes.c_int, ctypes.c_int, _P, _P, _P,
+                                    _P]),
+    "cg_graph_status": (ctypes.c_int, [_P, _P]),
     "cg_query_host": (ctypes.c_int, [_P, ctypes.c_int, _P, ctypes.c_int32, ctypes.c_int, _P, ctypes.c_int32, _P]),
+    "cg_query_host_fmt": (ctypes.c_int, [_P, ctypes.c_int, _P, ctypes.c_int32, ctypes.c_int, ctypes.c_int, _P,
+                                         ctypes.c_int32, _P]),
     "cg_rmat_generate": (ctypes.c_int, [ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32,
                                         ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int32, ctypes.c_uint64,
                                         ctypes.c_uint64, _P, _P, _P, _P]),

@@ -83,13 +83,42 @@ void check_sources_host(const Graph& G, const uint32_t* src, int32_t n_src) {
     for (int32_t i = 0; i < n_src; ++i) CGB_CHECK(src[i] < G.n, CG_EINVAL, "source id >= n");
 }
 
-__global__ void k_check_src(const uint32_t* __restrict__ src, int32_t n_src, uint32_t n, uint32_t* bad) {
-    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n_src; i += gridDim.x * blockDim.x)
-        if (src[i] >= n) atomicOr(bad, 1u);
+// the graph's sticky device error (graph.hpp), returned (and cleared) by the next call
+void take_sticky(Graph& G) {
+    if (!G.sticky_h) return;
+    volatile uint32_t* p = G.sticky_h;
+    const uint32_t e = *p;
+    if (!e) return;
+    *p = 0u;
+    CGB_CHECK(!(e & ERR_SOURCE), CG_EINVAL, "a source id >= n was passed to an asynchronous query (its row holds InitVal)");
+    CGB_CHECK(!(e & ERR_NARROW), CG_EOVERFLOW, "a value did not fit the requested narrow output format");
+    CGB_CHECK(!(e & ERR_ITERS), CG_EINTERNAL, "iteration bound exceeded");
+}
+
+// calls on one graph run in issue order across streams (they share the workspace)
+void order_begin(Graph& G, cudaStream_t s) {
+    if (G.last_valid && G.last_stream != s) CGB_CUDA(cudaStreamWaitEvent(s, G.last, 0));
+}
+void order_end(Graph& G, cudaStream_t s) {
+    CGB_CUDA(cudaEventRecord(G.last, s));
+    G.last_stream = s;
+    G.last_valid = true;
+}
+
+size_t row_bytes_of(const Graph& G, int fmt) {
+    return fmt == CG_OUT_U16 ? 2ull * G.n : fmt == CG_OUT_BITS ? 4ull * ((G.n + 31) / 32) : 4ull * G.n;
+}
+
+void check_format(int kind, int fmt) {
+    CGB_CHECK(fmt == CG_OUT_U32 || fmt == CG_OUT_U16 || fmt == CG_OUT_BITS, CG_EINVAL, "bad cg_out_format");
+    CGB_CHECK(fmt != CG_OUT_U16 || (kind != CG_VITERBI && kind != CG_WCC), CG_EINVAL,
+              "CG_OUT_U16 holds integer values: not for VITERBI or WCC");
+    CGB_CHECK(fmt != CG_OUT_BITS || kind == CG_REACH, CG_EINVAL, "CG_OUT_BITS is REACH's format");
 }
 
 void prepare_query(cg_graph g, int kind, int32_t n_src, int mode, const void* out, const uint32_t* src) {
     CGB_CHECK(g != nullptr, CG_EINVAL, "null graph");
+    take_sticky(g->G);
     check_kind(kind);
     CGB_CHECK(n_src >= 0, CG_EINVAL, "n_src < 0");
     CGB_CHECK(mode == CG_MODE_2PHASE || mode == CG_MODE_FULL, CG_EINVAL, "bad cg_mode");
@@ -134,6 +163,10 @@ cg_status cg_graph_create(int device, int64_t n, int64_t m, const uint32_t* src,
             h->G.device = device;
             h->stream = S(stream);
             CGB_CUDA(cudaDeviceGetAttribute(&h->G.num_sms, cudaDevAttrMultiProcessorCount, device));
+            CGB_CUDA(cudaHostAlloc(&h->G.sticky_h, sizeof(uint32_t), cudaHostAllocMapped));
+            *h->G.sticky_h = 0u;
+            CGB_CUDA(cudaHostGetDevicePointer((void**)&h->G.sticky_d, h->G.sticky_h, 0));
+            CGB_CUDA(cudaEventCreateWithFlags(&h->G.last, cudaEventDisableTiming));
             build_graph(h->G, n, m, src, dst, w, S(stream));
         } catch (...) {
             delete h;
@@ -148,6 +181,7 @@ cg_status cg_graph_destroy(cg_graph g) {
         if (!g) return;
         cudaSetDevice(g->G.device);
         cudaStreamSynchronize(g->stream);
+        if (g->G.last_valid) cudaEventSynchronize(g->G.last);
         delete g;
     });
 }
@@ -179,7 +213,9 @@ cg_status cg_build_ex(cg_graph g, cg_kind kind, int32_t K, cg_hub_policy policy,
         if (kind == CG_SSSP)
             CGB_CHECK((uint64_t)(g->G.n - 1) * g->G.w_max < 0xFFFFFFFFull, CG_EOVERFLOW,
                       "(n-1)*w_max >= 2^32-1: SSSP distances could wrap");
+        order_begin(g->G, S(stream));
         build_core(g->G, kind, K, policy, hubs, seed, alg, connectivity, S(stream));
+        order_end(g->G, S(stream));
     });
 }
 
@@ -194,7 +230,9 @@ cg_status cg_build_partial(cg_graph g, cg_kind kind, int32_t K, cg_hub_policy po
         CGB_CHECK(g != nullptr && (flags != nullptr || g->G.m == 0), CG_EINVAL, "null argument");
         check_kind(kind);
         CGB_CUDA(cudaSetDevice(g->G.device));
+        order_begin(g->G, S(stream));
         build_core_partial(g->G, kind, K, policy, hubs, seed, hub_begin, hub_end, flags, S(stream));
+        order_end(g->G, S(stream));
     });
 }
 
@@ -204,7 +242,9 @@ cg_status cg_build_from_flags(cg_graph g, cg_kind kind, int32_t K, cg_hub_policy
         CGB_CHECK(g != nullptr && (flags != nullptr || g->G.m == 0), CG_EINVAL, "null argument");
         check_kind(kind);
         CGB_CUDA(cudaSetDevice(g->G.device));
+        order_begin(g->G, S(stream));
         build_core_from_flags(g->G, kind, K, policy, hubs, seed, flags, connectivity, S(stream));
+        order_end(g->G, S(stream));
     });
 }
 
@@ -213,7 +253,9 @@ cg_status cg_core_save(cg_graph g, cg_kind kind, const char* path, void* stream)
         CGB_CHECK(g != nullptr && path != nullptr, CG_EINVAL, "null argument");
         check_kind(kind);
         CGB_CUDA(cudaSetDevice(g->G.device));
+        order_begin(g->G, S(stream));
         save_core(g->G, kind, path, S(stream));
+        order_end(g->G, S(stream));
     });
 }
 
@@ -222,7 +264,9 @@ cg_status cg_core_load(cg_graph g, cg_kind kind, const char* path, void* stream)
         CGB_CHECK(g != nullptr && path != nullptr, CG_EINVAL, "null argument");
         check_kind(kind);
         CGB_CUDA(cudaSetDevice(g->G.device));
+        order_begin(g->G, S(stream));
         load_core(g->G, kind, path, S(stream));
+        order_end(g->G, S(stream));
     });
 }
 
@@ -232,7 +276,7 @@ cg_status cg_core_info(cg_graph g, cg_kind kind, int64_t* m_cg, int32_t* K, uint
         check_kind(kind);
         const Core& C = g->G.core[core_slot(kind)];
         CGB_CHECK(C.built, CG_ENOCG, "Core Graph not built for this kind");
-        if (m_cg) *m_cg = C.adj.m;
+        if (m_cg) *m_cg = C.m_cg;
         if (K) *K = (int32_t)C.hubs.size();
         if (hubs) std::memcpy(hubs, C.hubs.data(), 4 * C.hubs.size());
         if (build_ms) *build_ms = C.build_ms;
@@ -246,57 +290,110 @@ cg_status cg_core_export(cg_graph g, cg_kind kind, uint8_t* flags, void* stream)
         const Core& C = g->G.core[core_slot(kind)];
         CGB_CHECK(C.built, CG_ENOCG, "Core Graph not built for this kind");
         CGB_CUDA(cudaSetDevice(g->G.device));
-        if (g->G.m)
-            CGB_CUDA(cudaMemcpyAsync(flags, C.flags.get(), g->G.m, cudaMemcpyDeviceToDevice, S(stream)));
+        export_core_flags(g->G, C, flags, S(stream));
+    });
+}
+
+}  // extern "C"
+
+namespace capi_internal {
+
+// the call's engine inputs: G (split rows of the kind's CG in 2Phase), CG, G minus CG
+QueryCall make_call(Graph& G, int kind, bool two, const uint32_t* src, int32_t n_src, void* out, uint32_t* p1,
+                    bool want_stats, int fmt) {
+    QueryCall c{};
+    c.kind = kind;
+    c.two_phase = two ? 1 : 0;
+    c.srcs = src;
+    c.n_src = n_src;
+    c.out = out;
+    c.p1 = two ? p1 : nullptr;
+    c.want_stats = want_stats;
+    c.out_fmt = fmt;
+    if (kind == CG_WCC) {  // G ∪ G^R, CG ∪ CG^R
+        c.full = view(G.gsym);
+        c.core = two ? view(G.core[CG_REACH].sym) : c.full;
+        c.rest = GraphView{};
+        c.cg = nullptr;
+        return c;
+    }
+    const Core& C = G.core[core_slot(kind)];
+    if (two) {
+        c.full = split_view(G, C);
+        c.core = core_view(G, C);
+        c.rest = rest_view(G, C);
+        c.cg = &C;
+    } else {
+        c.full = view(G.g);
+        c.core = c.full;
+        c.rest = GraphView{};
+        c.cg = nullptr;
+    }
+    return c;
+}
+
+}  // namespace capi_internal
+
+extern "C" {
+
+cg_status cg_query_fmt(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode, cg_out_format fmt,
+                       void* out, void* p1_out, cg_stats* stats, void* stream) {
+    return guard([&] {
+        prepare_query(g, kind, n_src, mode, out, src);
+        check_format(kind, fmt);
+        if (n_src == 0) return;
+        Graph& G = g->G;
+        CGB_CUDA(cudaSetDevice(G.device));
+        cudaStream_t s = S(stream);
+        order_begin(G, s);
+        if (kind == CG_WCC) src = nullptr;  // whole-graph query: no source
+        if (kind == CG_WCC) ensure_wcc_graphs(G, mode == CG_MODE_2PHASE, s);
+        const bool two = mode == CG_MODE_2PHASE;
+        QueryCall c = make_call(G, kind, two, src, n_src, out, (uint32_t*)p1_out, stats != nullptr, fmt);
+        std::vector<cg_stats> st;
+        run_queries(G, c, s, stats ? &st : nullptr);
+        order_end(G, s);
+        if (stats) {
+            CGB_CUDA(cudaStreamSynchronize(s));
+            take_sticky(G);  // this call's own device errors
+            std::memcpy(stats, st.data(), sizeof(cg_stats) * (size_t)n_src);
+        }
     });
 }
 
 cg_status cg_query_ex(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode, void* out,
                       void* p1_out, cg_stats* stats, void* stream) {
-    return guard([&] {
-        prepare_query(g, kind, n_src, mode, out, src);
-        if (n_src == 0) return;
-        Graph& G = g->G;
-        CGB_CUDA(cudaSetDevice(G.device));
-        if (kind == CG_WCC) src = nullptr;  // whole-graph query: no source
-        if (kind == CG_WCC) ensure_wcc_graphs(G, mode == CG_MODE_2PHASE, S(stream));
-        if (stats && src) {  // validate sources on device (the call synchronises anyway)
-            DevBuf<uint32_t> bad(1, S(stream));
-            CGB_CUDA(cudaMemsetAsync(bad.get(), 0, 4, S(stream)));
-            CGB_LAUNCH(k_check_src, 1, 256, 0, S(stream), src, n_src, G.n, bad.get());
-            uint32_t hb = 0;
-            CGB_CUDA(cudaMemcpyAsync(&hb, bad.get(), 4, cudaMemcpyDeviceToHost, S(stream)));
-            CGB_CUDA(cudaStreamSynchronize(S(stream)));
-            CGB_CHECK(!hb, CG_EINVAL, "source id >= n");
-        }
-        const bool two = mode == CG_MODE_2PHASE;
-        Adj* full = kind == CG_WCC ? &G.gsym : &G.g;
-        Adj* core = kind == CG_WCC ? &G.core[CG_REACH].sym : &G.core[core_slot(kind)].adj;
-        QueryCall c{(int)kind, full, two ? core : full, two ? 1 : 0, src, n_src,
-                    (uint32_t*)out, two ? (uint32_t*)p1_out : nullptr, stats != nullptr};
-        std::vector<cg_stats> st;
-        run_queries(G, c, S(stream), stats ? &st : nullptr);
-        if (stats) std::memcpy(stats, st.data(), sizeof(cg_stats) * (size_t)n_src);
-    });
+    return cg_query_fmt(g, kind, src, n_src, mode, CG_OUT_U32, out, p1_out, stats, stream);
 }
 
 cg_status cg_query(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode, void* out,
                    cg_stats* stats, void* stream) {
-    return cg_query_ex(g, kind, src, n_src, mode, out, nullptr, stats, stream);
+    return cg_query_fmt(g, kind, src, n_src, mode, CG_OUT_U32, out, nullptr, stats, stream);
 }
 
-cg_status cg_query_host(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode, void* out,
-                        int32_t batch, void* stream) {
+cg_status cg_graph_status(cg_graph g, void* stream) {
+    return guard([&] {
+        CGB_CHECK(g != nullptr, CG_EINVAL, "null graph");
+        CGB_CUDA(cudaSetDevice(g->G.device));
+        CGB_CUDA(cudaStreamSynchronize(S(stream)));
+        take_sticky(g->G);
+    });
+}
+
+cg_status cg_query_host_fmt(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode,
+                            cg_out_format fmt, void* out, int32_t batch, void* stream) {
     return guard([&] {
         prepare_query(g, kind, n_src, mode, out, src);
+        check_format(kind, fmt);
         if (n_src == 0) return;
         Graph& G = g->G;
         if (kind == CG_WCC) src = nullptr;
         if (src) check_sources_host(G, src, n_src);
         CGB_CUDA(cudaSetDevice(G.device));
         cudaStream_t s = S(stream);
+        order_begin(G, s);
         if (kind == CG_WCC) ensure_wcc_graphs(G, mode == CG_MODE_2PHASE, s);
-        const size_t row = (size_t)G.n * 4;
+        const size_t row = row_bytes_of(G, fmt);
         if (batch <= 0) {  // ~256 MiB of results per batch, at least 1 query
             size_t b = ((size_t)256 << 20) / (row ? row : 1);
             batch = (int32_t)(b < 1 ? 1 : (b > (size_t)n_src ? (size_t)n_src : b));
@@ -305,9 +402,9 @@ cg_status cg_query_host(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n
         DevBuf<uint32_t> dsrc((size_t)n_src, s);
         if (src) CGB_CUDA(cudaMemcpyAsync(dsrc.get(), src, 4ull * n_src, cudaMemcpyHostToDevice, s));
         // two result slots: batch b computes on `s` into slot b%2 while batch b-1 drains on `cp`
-        DevBuf<uint32_t> slot[2];
-        slot[0].alloc((size_t)batch * G.n, s);
-        if (n_src > batch) slot[1].alloc((size_t)batch * G.n, s);
+        DevBuf<uint8_t> slot[2];
+        slot[0].alloc((size_t)batch * row, s);
+        if (n_src > batch) slot[1].alloc((size_t)batch * row, s);
         cudaStream_t cp;
         CGB_CUDA(cudaStreamCreateWithFlags(&cp, cudaStreamNonBlocking));
         cudaEvent_t done[2], drained[2];
@@ -321,25 +418,30 @@ cg_status cg_query_host(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n
             const int32_t nq = (n_src - q0) < batch ? (n_src - q0) : batch;
             const int k = b & 1;
             if (b >= 2) CGB_CUDA(cudaStreamWaitEvent(s, drained[k], 0));
-            Adj* full = kind == CG_WCC ? &G.gsym : &G.g;
-            Adj* core = kind == CG_WCC ? &G.core[CG_REACH].sym : &G.core[core_slot(kind)].adj;
-            QueryCall c{(int)kind, full, two ? core : full, two ? 1 : 0, src ? dsrc.get() + q0 : nullptr,
-                        nq, slot[k].get(), nullptr, false};
+            QueryCall c = make_call(G, kind, two, src ? dsrc.get() + q0 : nullptr, nq, slot[k].get(), nullptr, false,
+                                    fmt);
             run_queries(G, c, s, nullptr);
             CGB_CUDA(cudaEventRecord(done[k], s));
             CGB_CUDA(cudaStreamWaitEvent(cp, done[k], 0));
-            CGB_CUDA(cudaMemcpyAsync((uint32_t*)out + (size_t)q0 * G.n, slot[k].get(), (size_t)nq * row,
+            CGB_CUDA(cudaMemcpyAsync((uint8_t*)out + (size_t)q0 * row, slot[k].get(), (size_t)nq * row,
                                      cudaMemcpyDeviceToHost, cp));
             CGB_CUDA(cudaEventRecord(drained[k], cp));
         }
         CGB_CUDA(cudaStreamSynchronize(cp));
         CGB_CUDA(cudaStreamSynchronize(s));
+        order_end(G, s);
         for (int i = 0; i < 2; ++i) {
             cudaEventDestroy(done[i]);
             cudaEventDestroy(drained[i]);
         }
         cudaStreamDestroy(cp);
+        take_sticky(G);
     });
+}
+
+cg_status cg_query_host(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode, void* out,
+                        int32_t batch, void* stream) {
+    return cg_query_host_fmt(g, kind, src, n_src, mode, CG_OUT_U32, out, batch, stream);
 }
 
 cg_status cg_rmat_generate(uint64_t n, uint32_t tA, uint32_t tAB, uint32_t tABC, uint32_t w_max, uint64_t seed,

@@ -148,41 +148,57 @@ __global__ void k_connectivity(uint32_t n, GraphView g, uint32_t dbits, int kind
     }
 }
 
-// ---------------------------------------------------------------- a7: compaction
-// (inv: count / scatter the UNflagged edges — G minus the CG, phase 2's first sweep)
-__global__ void k_row_count(uint32_t n, const uint32_t* __restrict__ ptr, const uint8_t* __restrict__ flags,
-                            uint32_t* __restrict__ cnt, int inv = 0) {
-    const uint32_t lane = threadIdx.x & 31;
-    const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
-    for (uint64_t u = blockIdx.x * (uint64_t)(blockDim.x / 32) + (threadIdx.x >> 5); u <= n; u += nw) {
-        if (u == n) { if (lane == 0) cnt[n] = 0; continue; }
-        uint32_t c = 0;
-        for (uint32_t e = ptr[u] + lane; e < ptr[u + 1]; e += 32) c += (flags[e] != 0) != (inv != 0);
-        for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(FULLM, c, o);
-        if (lane == 0) cnt[u] = c;
+// ---------------------------------------------------------------- a7: split rows
+// E_c membership bits (bit e of word e/32) from the u8 marks: thread per word, coalesced
+__global__ void k_pack_bits(uint64_t m, const uint8_t* __restrict__ flags, uint32_t* __restrict__ bits) {
+    for (uint64_t wi = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; wi < (m + 31) / 32;
+         wi += (uint64_t)gridDim.x * blockDim.x) {
+        uint32_t x = 0;
+        for (uint32_t b = 0; b < 32 && wi * 32 + b < m; ++b) x |= (uint32_t)(flags[wi * 32 + b] != 0) << b;
+        bits[wi] = x;
     }
 }
 
-__global__ void k_scatter_core(uint32_t n, const uint32_t* __restrict__ ptr, const uint8_t* __restrict__ flags,
-                               const uint32_t* __restrict__ cptr, const uint32_t* __restrict__ adj,
-                               const uint2* __restrict__ adjw, uint32_t* __restrict__ cadj, uint2* __restrict__ cadjw,
-                               int inv = 0) {
+__global__ void k_unpack_bits(uint64_t m, const uint32_t* __restrict__ bits, uint8_t* __restrict__ flags) {
+    for (uint64_t e = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; e < m; e += (uint64_t)gridDim.x * blockDim.x)
+        flags[e] = (bits[e >> 5] >> (e & 31)) & 1u;
+}
+
+__device__ __forceinline__ bool bit_at(const uint32_t* __restrict__ bits, uint32_t e) { return (bits[e >> 5] >> (e & 31)) & 1u; }
+
+// Split-CSR layout (graph.hpp Core): warp per row u of G; the row's CG edges are
+// copied to [ptr[u], cg_end[u]) and the others to [cg_end[u], ptr[u+1]), both in canonical
+// order (stable partition); *mcg accumulates |E_c|.
+__global__ void k_split_rows(uint32_t n, const uint32_t* __restrict__ ptr, const uint32_t* __restrict__ bits,
+                             const uint32_t* __restrict__ adj, const uint2* __restrict__ adjw,
+                             uint32_t* __restrict__ sadj, uint2* __restrict__ sadjw, uint32_t* __restrict__ cg_end,
+                             unsigned long long* __restrict__ mcg) {
     const uint32_t lane = threadIdx.x & 31;
+    const uint32_t lt = (1u << lane) - 1u;
     const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
+    unsigned long long tot = 0;
     for (uint64_t u = blockIdx.x * (uint64_t)(blockDim.x / 32) + (threadIdx.x >> 5); u < n; u += nw) {
-        uint32_t o = cptr[u];
         const uint32_t r0 = ptr[u], r1 = ptr[u + 1];
+        uint32_t c = 0;
+        for (uint32_t b = r0; b < r1; b += 32) c += __popc(__ballot_sync(FULLM, b + lane < r1 && bit_at(bits, b + lane)));
+        const uint32_t ce = r0 + c;
+        uint32_t oc = r0, orr = ce;
         for (uint32_t b = r0; b < r1; b += 32) {
             const uint32_t e = b + lane;
-            const bool f = e < r1 && ((flags[e] != 0) != (inv != 0));
-            const uint32_t bal = __ballot_sync(FULLM, f);
-            if (f) {
-                const uint32_t p = o + __popc(bal & ((1u << lane) - 1u));
-                if (adj) cadj[p] = adj[e]; else cadjw[p] = adjw[e];
+            const bool in = e < r1;
+            const bool f = in && bit_at(bits, e);
+            const uint32_t bc = __ballot_sync(FULLM, f), br = __ballot_sync(FULLM, in && !f);
+            if (in) {
+                const uint32_t p = f ? oc + __popc(bc & lt) : orr + __popc(br & lt);
+                if (adj) sadj[p] = adj[e]; else sadjw[p] = adjw[e];
             }
-            o += __popc(bal);
+            oc += __popc(bc);
+            orr += __popc(br);
         }
+        if (lane == 0) cg_end[u] = ce;
+        tot += c;
     }
+    if (lane == 0 && tot) atomicAdd(mcg, tot);
 }
 
 // ---------------------------------------------------------------- a5': Alg 2
@@ -337,9 +353,11 @@ void alg1(Graph& G, int kind, const std::vector<uint32_t>& hubs, uint8_t* flags,
     DevBuf<uint32_t> vf((size_t)group * G.n, s), vb((size_t)group * G.n, s);
     for (int k0 = 0; k0 < K; k0 += group) {
         const int nh = (K - k0) < group ? (K - k0) : group;
-        QueryCall f{kind, &G.g, &G.g, 0, hsrc.get() + k0, nh, vf.get(), nullptr, false};
+        QueryCall f{kind, view(G.g), view(G.g), GraphView{}, nullptr, 0, hsrc.get() + k0, nh, vf.get(), nullptr,
+                    false, CG_OUT_U32};
         run_queries(G, f, s, nullptr);                   // Alg 1 l.4: Identify(G, forward)
-        QueryCall b{kind, &G.gr, &G.gr, 0, hsrc.get() + k0, nh, vb.get(), nullptr, false};
+        QueryCall b{kind, view(G.gr), view(G.gr), GraphView{}, nullptr, 0, hsrc.get() + k0, nh, vb.get(), nullptr,
+                    false, CG_OUT_U32};
         run_queries(G, b, s, nullptr);                   // Alg 1 l.5: Identify(G^R, backward)
         switch (kind) {
         case CG_SSSP: mark_group<CG_SSSP>(G, nh, vf.get(), vb.get(), flags, s); break;
@@ -410,39 +428,32 @@ void alg2(Graph& G, const std::vector<uint32_t>& hubs, uint8_t* flags, bool per_
 
 namespace {
 
-// a6 + a7: connectivity edges (Alg 1 l.8-12) on C.flags, then stream compaction into C.adj
-void finalize_core(Graph& G, int kind, Core& C, int connectivity, cudaStream_t s) {
+// a7: the split rows from C.fbits
+void split_core(Graph& G, Core& C, cudaStream_t s) {
+    C.cg_end.alloc(G.n ? G.n : 1, s);
+    C.sadj.reset();
+    C.sadjw.reset();
+    if (G.packed) C.sadj.alloc(adj_alloc_elems(G.m, 4), s); else C.sadjw.alloc(adj_alloc_elems(G.m, 8), s);
+    DevBuf<unsigned long long> mcg(1, s);
+    CGB_CUDA(cudaMemsetAsync(mcg.get(), 0, 8, s));
+    CGB_LAUNCH(k_split_rows, grid_rows(G.n), TB, 0, s, G.n, G.g.ptr.get(), C.fbits.get(), G.g.adj.get(), G.g.adjw.get(),
+               C.sadj.get(), C.sadjw.get(), C.cg_end.get(), mcg.get());
+    unsigned long long h = 0;
+    CGB_CUDA(cudaMemcpyAsync(&h, mcg.get(), 8, cudaMemcpyDeviceToHost, s));
+    CGB_CUDA(cudaStreamSynchronize(s));
+    C.m_cg = (uint32_t)h;
+}
+
+// a6 + a7: connectivity edges (Alg 1 l.8-12) on the u8 marks (device, m bytes, consumed),
+// then the membership bitmap and the split rows (graph.hpp Core)
+void finalize_core(Graph& G, int kind, Core& C, int connectivity, uint8_t* marks, cudaStream_t s) {
     if (G.m && connectivity) {
         const int sel = (kind == CG_SSWP) ? 1 : ((kind == CG_BFS || kind == CG_REACH) ? 2 : 0);
-        CGB_LAUNCH(k_connectivity, grid_rows(G.n), TB, 0, s, G.n, view(G.g), G.dbits, sel, C.flags.get());
+        CGB_LAUNCH(k_connectivity, grid_rows(G.n), TB, 0, s, G.n, view(G.g), G.dbits, sel, marks);
     }
-    DevBuf<uint32_t> cnt(G.n + 1, s);
-    C.adj.n = G.n;
-    C.adj.ptr.alloc(G.n + 1, s);
-    CGB_LAUNCH(k_row_count, grid_rows(G.n + 1), TB, 0, s, G.n, G.g.ptr.get(), C.flags.get(), cnt.get());
-    exclusive_sum(cnt.get(), C.adj.ptr.get(), (uint64_t)G.n + 1, s);
-    uint32_t mcg = 0;
-    CGB_CUDA(cudaMemcpyAsync(&mcg, C.adj.ptr.get() + G.n, 4, cudaMemcpyDeviceToHost, s));
-    CGB_CUDA(cudaStreamSynchronize(s));
-    C.adj.m = mcg;
-    C.adj.adj.reset();
-    C.adj.adjw.reset();
-    if (G.packed) C.adj.adj.alloc(adj_alloc_elems(mcg, 4), s); else C.adj.adjw.alloc(adj_alloc_elems(mcg, 8), s);
-    CGB_LAUNCH(k_scatter_core, grid_rows(G.n), TB, 0, s, G.n, G.g.ptr.get(), C.flags.get(), C.adj.ptr.get(),
-               G.g.adj.get(), G.g.adjw.get(), C.adj.adj.get(), C.adj.adjw.get(), 0);
-    // G minus the CG (reading N7, the split-CSR benefit P:2567-2572): after phase 1 every CG
-    // edge is at its fixpoint, so phase 2's first sweep relaxes only these edges
-    C.rest.n = G.n;
-    C.rest.ptr.alloc(G.n + 1, s);
-    CGB_LAUNCH(k_row_count, grid_rows(G.n + 1), TB, 0, s, G.n, G.g.ptr.get(), C.flags.get(), cnt.get(), 1);
-    exclusive_sum(cnt.get(), C.rest.ptr.get(), (uint64_t)G.n + 1, s);
-    C.rest.m = G.m - mcg;
-    C.rest.adj.reset();
-    C.rest.adjw.reset();
-    if (G.packed) C.rest.adj.alloc(adj_alloc_elems(C.rest.m, 4), s); else C.rest.adjw.alloc(adj_alloc_elems(C.rest.m, 8), s);
-    CGB_LAUNCH(k_scatter_core, grid_rows(G.n), TB, 0, s, G.n, G.g.ptr.get(), C.flags.get(), C.rest.ptr.get(),
-               G.g.adj.get(), G.g.adjw.get(), C.rest.adj.get(), C.rest.adjw.get(), 1);
-    C.rest_built = true;
+    C.fbits.alloc(((size_t)G.m + 31) / 32 + 1, s);
+    if (G.m) CGB_LAUNCH(k_pack_bits, 4 * G.num_sms, TB, 0, s, (uint64_t)G.m, marks, C.fbits.get());
+    split_core(G, C, s);
 }
 
 struct Timer {
@@ -528,13 +539,13 @@ void build_core(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs_
     C.sym_built = false;
     C.hub_vals.reset();
     C.hub_k = 0;
-    C.flags.alloc(G.m ? G.m : 1, s);
-    CGB_CUDA(cudaMemsetAsync(C.flags.get(), 0, C.flags.bytes(), s));
+    DevBuf<uint8_t> marks(G.m ? G.m : 1, s);  // E_c marks in G's CSR order (u8: racing writers)
+    CGB_CUDA(cudaMemsetAsync(marks.get(), 0, marks.bytes(), s));
     if (G.m) {
-        if (alg == CG_ALG_SPECIALIZED) alg1(G, kind, hubs, C.flags.get(), C, s);
-        else alg2(G, hubs, C.flags.get(), alg == CG_ALG_GENERAL_PERDIR, s);
+        if (alg == CG_ALG_SPECIALIZED) alg1(G, kind, hubs, marks.get(), C, s);
+        else alg2(G, hubs, marks.get(), alg == CG_ALG_GENERAL_PERDIR, s);
     }
-    finalize_core(G, kind, C, connectivity, s);
+    finalize_core(G, kind, C, connectivity, marks.get(), s);
     C.hubs = hubs;
     C.alg = alg;
     C.connectivity = connectivity;
@@ -547,7 +558,7 @@ void build_core(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs_
 // in-edges (G^R row v; an in-edge's flag is that of its CSR edge, reid).  Edge words keep G's
 // encoding (the WCC EdgeFunction ignores the weight).
 __global__ void k_sym_count(uint32_t n, const uint32_t* __restrict__ gp, const uint32_t* __restrict__ rp,
-                            const uint32_t* __restrict__ reid, const uint8_t* __restrict__ flags,
+                            const uint32_t* __restrict__ reid, const uint32_t* __restrict__ flags,
                             uint32_t* __restrict__ cnt) {
     const uint32_t lane = threadIdx.x & 31;
     const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
@@ -555,8 +566,8 @@ __global__ void k_sym_count(uint32_t n, const uint32_t* __restrict__ gp, const u
         if (u == n) { if (lane == 0) cnt[n] = 0; continue; }
         uint32_t c = 0;
         if (flags) {
-            for (uint32_t e = gp[u] + lane; e < gp[u + 1]; e += 32) c += flags[e] != 0;
-            for (uint32_t e = rp[u] + lane; e < rp[u + 1]; e += 32) c += flags[reid[e]] != 0;
+            for (uint32_t e = gp[u] + lane; e < gp[u + 1]; e += 32) c += bit_at(flags, e);
+            for (uint32_t e = rp[u] + lane; e < rp[u + 1]; e += 32) c += bit_at(flags, reid[e]);
             for (int o = 16; o > 0; o >>= 1) c += __shfl_xor_sync(FULLM, c, o);
         } else {
             c = (gp[u + 1] - gp[u]) + (rp[u + 1] - rp[u]);
@@ -566,13 +577,13 @@ __global__ void k_sym_count(uint32_t n, const uint32_t* __restrict__ gp, const u
 }
 
 __device__ __forceinline__ void sym_copy_row(uint32_t r0, uint32_t r1, const uint32_t* __restrict__ reid,
-                                             const uint8_t* __restrict__ flags, const uint32_t* __restrict__ adj,
+                                             const uint32_t* __restrict__ flags, const uint32_t* __restrict__ adj,
                                              const uint2* __restrict__ adjw, uint32_t* __restrict__ sadj,
                                              uint2* __restrict__ sadjw, uint32_t& o) {
     const uint32_t lane = threadIdx.x & 31;
     for (uint32_t b = r0; b < r1; b += 32) {
         const uint32_t e = b + lane;
-        const bool f = e < r1 && (!flags || flags[reid ? reid[e] : e]);
+        const bool f = e < r1 && (!flags || bit_at(flags, reid ? reid[e] : e));
         const uint32_t bal = __ballot_sync(FULLM, f);
         if (f) {
             const uint32_t p = o + __popc(bal & ((1u << lane) - 1u));
@@ -583,7 +594,7 @@ __device__ __forceinline__ void sym_copy_row(uint32_t r0, uint32_t r1, const uin
 }
 
 __global__ void k_sym_scatter(uint32_t n, const uint32_t* __restrict__ gp, const uint32_t* __restrict__ rp,
-                              const uint32_t* __restrict__ reid, const uint8_t* __restrict__ flags,
+                              const uint32_t* __restrict__ reid, const uint32_t* __restrict__ flags,
                               const uint32_t* __restrict__ sp, const uint32_t* __restrict__ gadj,
                               const uint2* __restrict__ gadjw, const uint32_t* __restrict__ radj,
                               const uint2* __restrict__ radjw, uint32_t* __restrict__ sadj, uint2* __restrict__ sadjw) {
@@ -595,7 +606,7 @@ __global__ void k_sym_scatter(uint32_t n, const uint32_t* __restrict__ gp, const
     }
 }
 
-void symmetrize(Graph& G, const uint8_t* flags, Adj& out, cudaStream_t s) {
+void symmetrize(Graph& G, const uint32_t* flags, Adj& out, cudaStream_t s) {
     DevBuf<uint32_t> cnt(G.n + 1, s);
     CGB_LAUNCH(k_sym_count, grid_rows(G.n + 1), TB, 0, s, G.n, G.g.ptr.get(), G.gr.ptr.get(), G.reid.get(), flags,
                cnt.get());
@@ -622,7 +633,7 @@ void ensure_wcc_graphs(Graph& G, bool two_phase, cudaStream_t s) {
     }
     Core& C = G.core[CG_REACH];
     if (two_phase && C.built && !C.sym_built) {
-        symmetrize(G, C.flags.get(), C.sym, s);
+        symmetrize(G, C.fbits.get(), C.sym, s);
         C.sym_built = true;
     }
 }
@@ -658,9 +669,9 @@ void build_core_from_flags(Graph& G, int kind, int32_t K, int policy, const uint
     C.sym_built = false;
     C.hub_vals.reset();
     C.hub_k = 0;
-    C.flags.alloc(G.m ? G.m : 1, s);
-    if (G.m) CGB_CUDA(cudaMemcpyAsync(C.flags.get(), flags, G.m, cudaMemcpyDeviceToDevice, s));
-    finalize_core(G, kind, C, connectivity, s);
+    DevBuf<uint8_t> marks(G.m ? G.m : 1, s);  // writable copy (connectivity edges are added)
+    if (G.m) CGB_CUDA(cudaMemcpyAsync(marks.get(), flags, G.m, cudaMemcpyDeviceToDevice, s));
+    finalize_core(G, kind, C, connectivity, marks.get(), s);
     C.hubs = hubs;
     C.alg = CG_ALG_SPECIALIZED;
     C.connectivity = connectivity;
@@ -674,12 +685,10 @@ void build_core_from_flags(Graph& G, int kind, int32_t K, int policy, const uint
 void save_core(Graph& G, int kind, const char* path, cudaStream_t s) {
     const Core& C = G.core[core_slot(kind)];
     CGB_CHECK(C.built, CG_ENOCG, "Core Graph not built for this kind");
-    std::vector<uint8_t> f(G.m);
-    if (G.m) CGB_CUDA(cudaMemcpyAsync(f.data(), C.flags.get(), G.m, cudaMemcpyDeviceToHost, s));
-    const unsigned long long h = graph_hash(G, s);
-    std::vector<uint8_t> bits((G.m + 7) / 8, 0);
-    for (size_t i = 0; i < f.size(); ++i)
-        if (f[i]) bits[i >> 3] |= (uint8_t)(1u << (i & 7));
+    // membership bits: bit e of word e/32 is, on this little-endian host, bit (e % 8) of byte e/8
+    std::vector<uint8_t> bits(((size_t)G.m + 7) / 8, 0);
+    if (G.m) CGB_CUDA(cudaMemcpyAsync(bits.data(), C.fbits.get(), bits.size(), cudaMemcpyDeviceToHost, s));
+    const unsigned long long h = graph_hash(G, s);  // (synchronises s)
     CoreFileHeader hd{};
     std::memcpy(hd.magic, kMagic, 8);
     hd.version = 1;
@@ -690,7 +699,7 @@ void save_core(Graph& G, int kind, const char* path, cudaStream_t s) {
     hd.n = G.n;
     hd.m = G.m;
     hd.graph_hash = h;
-    hd.m_cg = C.adj.m;
+    hd.m_cg = C.m_cg;
     FILE* fp = std::fopen(path, "wb");
     CGB_CHECK(fp != nullptr, CG_EINVAL, std::string("cannot open for writing: ") + path);
     bool ok = std::fwrite(&hd, sizeof hd, 1, fp) == 1;
@@ -715,23 +724,27 @@ void load_core(Graph& G, int kind, const char* path, cudaStream_t s) {
               "the file holds the Core Graph of another kind");
     CGB_CHECK(hd.n == G.n && hd.m == G.m && hd.graph_hash == graph_hash(G, s), CG_EINVAL,
               "the file was saved for another graph (n, m or fingerprint differ)");
+    if (G.m % 8) bits.back() &= (uint8_t)((1u << (G.m % 8)) - 1u);  // no stray bits past edge m-1
     Timer t(s);
-    std::vector<uint8_t> f(G.m);
-    for (size_t i = 0; i < f.size(); ++i) f[i] = (bits[i >> 3] >> (i & 7)) & 1u;
     Core& C = G.core[core_slot(kind)];
     C.built = false;
     C.sym_built = false;
     C.hub_vals.reset();
     C.hub_k = 0;
-    C.flags.alloc(G.m ? G.m : 1, s);
-    if (G.m) CGB_CUDA(cudaMemcpyAsync(C.flags.get(), f.data(), G.m, cudaMemcpyHostToDevice, s));
-    finalize_core(G, kind, C, 0, s);  // the saved flags already hold the connectivity edges
-    CGB_CHECK(C.adj.m == hd.m_cg, CG_EINVAL, "Core Graph file is inconsistent (edge count)");
+    C.fbits.alloc(((size_t)G.m + 31) / 32 + 1, s);
+    CGB_CUDA(cudaMemsetAsync(C.fbits.get(), 0, C.fbits.bytes(), s));
+    if (G.m) CGB_CUDA(cudaMemcpyAsync(C.fbits.get(), bits.data(), bits.size(), cudaMemcpyHostToDevice, s));
+    split_core(G, C, s);  // the saved bits already hold the connectivity edges
+    CGB_CHECK(C.m_cg == hd.m_cg, CG_EINVAL, "Core Graph file is inconsistent (edge count)");
     C.hubs = hubs;
     C.alg = (int)hd.alg;
     C.connectivity = (int)hd.connectivity;
     C.build_ms = t.stop();
     C.built = true;
+}
+
+void export_core_flags(Graph& G, const Core& C, uint8_t* flags, cudaStream_t s) {
+    if (G.m) CGB_LAUNCH(k_unpack_bits, 4 * G.num_sms, TB, 0, s, (uint64_t)G.m, C.fbits.get(), flags);
 }
 
 }  // namespace cgb

@@ -44,9 +44,9 @@ constexpr int S_PIPE = CGB_STAGES;  // value-row pipeline depth (chunks of 32 ed
 #endif
 constexpr int E_AHEAD = CGB_EAHEAD;  // edge-word lead over the row requests (chunks)
 
-enum { ST_IT1, ST_IT2, ST_E1, ST_E2, ST_U1, ST_U2, ST_F1, ST_F2, ST_IMP, ST_REACH, ST_PREC, ST_S1, ST_S2, NSTAT };
+enum { ST_IT1, ST_IT2, ST_E1, ST_E2, ST_U1, ST_U2, ST_F1, ST_F2, ST_IMP, ST_REACH, ST_PREC, ST_S1, ST_S2, ST_T1, ST_T2,
+       NSTAT };
 enum { CT0 = 8, CTS = 3, CT_LIST = 0, CT_ACTIVE = 1, CT_TILE = 2 };
-enum { ERR_ITERS = 1u, ERR_SOURCE = 2u, ERR_LANE_OVERFLOW = 4u };
 
 struct BParams {
     uint32_t n, words, dbits, dmask;
@@ -54,8 +54,9 @@ struct BParams {
     const uint32_t* srcs;
     int32_t n_src;
     int two_phase;
-    uint32_t* out;              // caller layout: out[q * n + v]
-    uint32_t* p1;               // nullable, caller layout
+    void* out;                  // caller layout: row q of n values in out_fmt (cg_out_format)
+    uint32_t* p1;               // nullable, caller layout (u32)
+    int out_fmt;
     uint32_t* V;                // [n][RW] value rows
     uint32_t* M;                // [n] active-query masks
     uint32_t* bitmap;           // [words] union frontier
@@ -64,12 +65,13 @@ struct BParams {
     uint32_t* lm;
     unsigned long long* ctrl;   // [0] barrier; [CT0 + CTS*slot + k] per-iteration counters
     unsigned long long* stats;  // nullable: per query NSTAT counters
-    uint32_t* err;
+    uint32_t* err;              // this call's lane-overflow word (ERR_LANE_OVERFLOW)
+    uint32_t* err_map;          // the graph's sticky error word (host-mapped): ERR_SOURCE / ERR_ITERS / ERR_NARROW
+    const uint32_t* guard;      // non-null: run only if *guard has ERR_LANE_OVERFLOW (the u32-lane re-run)
     uint32_t max_iters;
     uint32_t bits_below;        // frontiers smaller than this keep a bitmap (else the masks M are scanned)
     GraphView R;                // G^R: in-edges for the NEXT-1 pull
-    GraphView Rst;              // G minus the CG: phase 2's first sweep (reading N7)
-    int use_rest;
+    GraphView Rst;              // G minus the CG: phase 2's first sweep (reading N7); ptr null: G
     int dyn;                    // S2's second half in dynamically taken tiles
     const uint32_t* HB;         // CG hub rows [n][2K] for the certificates (nullable; u32 lanes only)
     uint32_t K, KP;             // hubs in HB; row stride 2*KP (KP = K rounded up to a multiple of 4)
@@ -502,6 +504,20 @@ __device__ __forceinline__ void span_loads(const BParams& P, const GraphView& g,
                                            uint32_t (&mv)[16], uint32_t (&dg)[16]) {
     const uint32_t lane = threadIdx.x & 31;
     uint32_t pv[16];
+    if (g.end) {  // split rows: [ptr[v], end[v])
+#pragma unroll
+        for (int j = 0; j < 16; ++j) {
+            const uint32_t wj = g0 + h * 16 + j;
+            const uint32_t v = wj * 32 + lane;
+            const bool ok = wj < w1 && v < P.n;
+            mv[j] = ok ? ld_cg(P.M + v) : 0u;
+            pv[j] = ok ? __ldg(g.ptr + v) : 0u;
+            dg[j] = ok ? __ldg(g.end + v) : 0u;
+        }
+#pragma unroll
+        for (int j = 0; j < 16; ++j) dg[j] = mv[j] ? dg[j] - pv[j] : 0u;
+        return;
+    }
 #pragma unroll
     for (int j = 0; j < 16; ++j) {
         const uint32_t wj = g0 + h * 16 + j;
@@ -1091,6 +1107,58 @@ __device__ void transpose_out(const BParams& P, uint32_t* dst, int q0, int nq, u
     }
 }
 
+// Narrow output formats (cg_out_format): the same values, fewer bytes on the wire.
+//   CG_OUT_U16:  row q = n uint16 values, InitVal / SourceInitVal 0xFFFFFFFF as 0xFFFF; a value
+//                >= 0xFFFF that is not 0xFFFFFFFF cannot be represented (ERR_NARROW -> CG_EOVERFLOW)
+//   CG_OUT_BITS: REACH only, row q = ceil(n/32) words, bit (v % 32) of word v / 32 = Val(v)
+// 32 vertices (a tile) per warp: the tile's rows through the padded shared tile (U16), or the
+// 32 x 32 bit matrix of a REACH tile transposed with one ballot per query (BITS).
+template <class L>
+__device__ void transpose_narrow(const BParams& P, int q0, int nq, uint32_t* xs) {
+    constexpr int RW = L::RW;
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t gw = blockIdx.x * BW + (threadIdx.x >> 5);
+    const uint32_t NW = gridDim.x * BW;
+    const uint32_t T = (P.n + 31) / 32;  // tiles
+    if constexpr (L::QPW == 32) {  // bit lanes: CG_OUT_BITS (the host admits REACH's bit lanes only)
+        if (P.out_fmt != CG_OUT_BITS) return;
+        uint32_t* dst = static_cast<uint32_t*>(P.out);
+        for (uint32_t tile = gw; tile < T; tile += NW) {
+            const uint32_t v = tile * 32 + lane;
+            const uint32_t row = v < P.n ? ld_cg(P.V + v) : 0u;
+            uint32_t mine = 0;
+            for (int q = 0; q < nq; ++q) {
+                const uint32_t b = __ballot_sync(FULL, (row >> q) & 1u);
+                if ((int)lane == q) mine = b;
+            }
+            if ((int)lane < nq) __stcs(dst + (size_t)(q0 + lane) * T + tile, mine);
+        }
+        return;
+    }
+    if (P.out_fmt != CG_OUT_U16) return;
+    uint16_t* dst = static_cast<uint16_t*>(P.out);
+    bool over = false;
+    for (uint32_t tile = gw; tile < T; tile += NW) {
+        __syncwarp();
+#pragma unroll
+        for (int r = 0; r < RW; ++r) {
+            const uint32_t f = r * 32 + lane;
+            const uint32_t v = tile * 32 + f / RW;
+            xs[(f / RW) * (RW + 1) + f % RW] = v < P.n ? __ldcg(P.V + (size_t)v * RW + f % RW) : 0u;
+        }
+        __syncwarp();
+        const uint32_t v = tile * 32 + lane;
+        if (v < P.n)
+            for (int q = 0; q < nq; ++q) {
+                const uint32_t x = L::decode(xs[lane * (RW + 1) + q / L::QPW], q % L::QPW);
+                over |= x >= 0xffffu && x != 0xffffffffu;
+                __stcs(reinterpret_cast<unsigned short*>(dst + (size_t)(q0 + q) * P.n + v),
+                       (unsigned short)(x >= 0xffffu ? 0xffffu : x));
+            }
+    }
+    if (over) atomicOr(P.err, ERR_NARROW);
+}
+
 template <class L>  // per warp, 16 B aligned: one or two 32-row windows (S2) or the padded transpose tile
 constexpr uint32_t xs_words() {
     return (xs_double<L>() ? 2 : 1) * 32 * L::RW > ((32 * (L::RW + 1) + 3) & ~3u) ? (xs_double<L>() ? 2 : 1) * 32 * L::RW
@@ -1110,16 +1178,25 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
     uint32_t* xs = dsm + (threadIdx.x >> 5) * xs_words<L>();
     uint32_t* vs = dsm + BW * xs_words<L>() + (threadIdx.x >> 5) * vs_words<L>();
     uint32_t* sh = dsm + BW * (xs_words<L>() + vs_words<L>());
+    // the u32-lane re-run of a binary16 call (reading N3) runs only if that call overflowed;
+    // every CTA reads the same word, so the whole grid exits together
+    if (P.guard && !(ld_cg(P.guard) & ERR_LANE_OVERFLOW)) return;
     unsigned long long epoch = 0;
     const uint64_t tid = blockIdx.x * (uint64_t)BT + threadIdx.x;
     const uint64_t nthreads = (uint64_t)gridDim.x * BT;
     uint32_t ring = 0;
+    // thread 0's bookkeeping lives in shared memory (not registers live across the loop):
+    // sticky errors of this launch, and the pass's start / phase-switch times (stats)
+    __shared__ uint32_t sm_err;
+    __shared__ unsigned long long sm_t[2];
+    if (threadIdx.x == 0) sm_err = 0u;
 
     // kernel-level trace marks (tid 0): [cap-1] = {entry, seeds done, loop done, exit} of batch 0
     unsigned long long* kt = (P.trace && tid == 0) ? P.trace + 5ull * (P.trace_cap - 1) : nullptr;
     if (kt) kt[0] = global_ns();
     for (int q0 = 0; q0 < P.n_src; q0 += Q) {
         const int nq = min(Q, P.n_src - q0);
+        if (P.stats && tid == 0) sm_t[0] = sm_t[1] = global_ns();
         // Alg 3 l.4, l.6 for every query of the batch; masks cleared
         if constexpr (RW % 4 == 0 && !InitOf<L>::ALL_ACTIVE) {  // 16 B stores
             const uint32_t iw = L::init_word();
@@ -1133,8 +1210,8 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
         grid_sync(P.ctrl, epoch);
         for (int b = 0; b < nq && !InitOf<L>::ALL_ACTIVE; ++b) {
             const uint32_t s = __ldg(P.srcs + q0 + b);
-            if (s >= P.n) {
-                if (tid == 0) atomicOr(P.err, ERR_SOURCE);
+            if (s >= P.n) {  // CG_EINVAL, reported through the sticky word; the row stays InitVal
+                if (threadIdx.x == 0) sm_err |= ERR_SOURCE;
                 continue;
             }
             uint32_t* col = P.V + b / L::QPW;
@@ -1170,7 +1247,7 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
         for (;;) {
             // phase 2's first sweep (Alg 3 l.15 seeding, `predicate`) relaxes G minus the CG:
             // every CG edge is at its fixpoint after phase 1 (reading N7)
-            const GraphView& g = (phase == 1) ? P.C : (predicate && P.use_rest) ? P.Rst : P.G;
+            const GraphView& g = (phase == 1) ? P.C : (predicate && P.Rst.ptr) ? P.Rst : P.G;
             const bool fresh = (P.fresh >> (phase - 1)) & 1u;
             const int slot = ring & 3;
             unsigned long long* ctr = P.ctrl + CT0 + CTS * slot;
@@ -1234,6 +1311,7 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
                     }
                     // the p1 / impacted reads must finish before phase 2 updates V
                     if (P.p1 || P.stats) grid_sync(P.ctrl, epoch);
+                    if (P.stats && tid == 0) sm_t[1] = global_ns();
                     phase = 2;
                     if (P.reduced) pull = true;   // Reduced(E): pull into uncertified vertices
                     else predicate = true;        // Active <- impacted vertices (l.15)
@@ -1263,13 +1341,18 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
             }
             grid_sync(P.ctrl, epoch);
             if (P.trace && tid == 0 && tr + 1 < P.trace_cap) P.trace[5ull * tr + 2] = global_ns();
-            if (++iters > P.max_iters) {
-                if (tid == 0) atomicOr(P.err, ERR_ITERS);
+            if (++iters > P.max_iters) {  // cannot happen for a monotone fixpoint; every CTA agrees
+                if (tid == 0) report_sticky(P.err_map, sm_err | ERR_ITERS);
                 return;
             }
         }
         if (kt && q0 == 0) kt[2] = global_ns();
-        transpose_out<L>(P, P.out, q0, nq, xs, vs);
+        if constexpr (KIND == CG_VITERBI || KIND == CG_WCC) {  // u32 only (the host rejects the others)
+            transpose_out<L>(P, static_cast<uint32_t*>(P.out), q0, nq, xs, vs);
+        } else {
+            if (P.out_fmt == CG_OUT_U32) transpose_out<L>(P, static_cast<uint32_t*>(P.out), q0, nq, xs, vs);
+            else transpose_narrow<L>(P, q0, nq, xs);
+        }
         if (P.stats) {  // reached / precise per query (the thread's query q is fixed)
             const uint32_t q = (uint32_t)(tid % Q);
             const uint32_t sb = ((int)q < nq && P.srcs) ? __ldg(P.srcs + q0 + q) : 0xffffffffu;
@@ -1287,8 +1370,18 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
             per_query_add<Q>(P.stats, q0, nq, ST_PREC, pr);
         }
         grid_sync(P.ctrl, epoch);  // V / M / bitmap are reused by the next batch
+        if (P.stats && tid == 0) {  // device time of this pass's phases, for each of its queries
+            const unsigned long long t_end = global_ns();
+            for (int b = 0; b < nq; ++b) {
+                atomicAdd(P.stats + (size_t)(q0 + b) * NSTAT + ST_T1, sm_t[1] - sm_t[0]);
+                atomicAdd(P.stats + (size_t)(q0 + b) * NSTAT + ST_T2, t_end - sm_t[1]);
+            }
+        }
     }
     if (kt) kt[3] = global_ns();
+    // sticky errors: a bad source (seen by every thread), a narrow-output overflow (any thread,
+    // collected in P.err; the pass's final grid barrier made it visible)
+    if (tid == 0) report_sticky(P.err_map, sm_err | (ld_cg(P.err) & ERR_NARROW));
 }
 
 template <int KIND, bool PACKED, int LW>
@@ -1355,8 +1448,11 @@ int lane_width(const Graph& G, int kind) {
     return 32;
 }
 
+// One launch of the batched kernel for the call.  guard != null: the u32-lane re-run of a
+// binary16 call, which executes only if that call set ERR_LANE_OVERFLOW in *guard (the per-call
+// word is then not cleared).
 void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::vector<cg_stats>* stats,
-                    uint32_t* err_out) {
+                    const uint32_t* guard) {
     BatchSpace& w = G.bs;
     const uint32_t words = (G.n + 31) / 32;
     if (w.n != G.n) {
@@ -1379,8 +1475,8 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
     P.words = words;
     P.dbits = G.dbits;
     P.dmask = G.dbits >= 32 ? 0xffffffffu : ((1u << G.dbits) - 1u);
-    P.G = view(*c.full_adj);
-    P.C = c.two_phase ? view(*c.core_adj) : P.G;
+    P.G = c.full;
+    P.C = c.two_phase ? c.core : c.full;
     P.R = view(G.gr);
     {   // NEXT-1 (Reduced(E) pull) after phase 1 for the kinds with a certificate; CG_REDUCED is a
         // bitmask over cg_kind.  Default REACH only: its certificate (reached = final) leaves only
@@ -1390,14 +1486,15 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
         const char* e = getenv("CG_REDUCED");
         const unsigned mask = e ? (unsigned)strtoul(e, nullptr, 0) : (1u << CG_REACH);
         const Core& core = G.core[core_slot(c.kind)];
+        const bool kind_cg = c.two_phase && c.cg == &core;
         const bool hub_cert = lw == 32 && core.hub_k > 0 && core.hub_k <= 64 && core.hub_vals.get();
         const bool has_cert = c.kind == CG_REACH || hub_cert;
-        P.reduced = c.two_phase && c.core_adj == &core.adj && ((mask >> c.kind) & 1u) && has_cert;
+        P.reduced = kind_cg && ((mask >> c.kind) & 1u) && has_cert;
         const char* dy = getenv("CG_DYN");
         P.dyn = dy ? atoi(dy) : 1;
         const char* rs = getenv("CG_REST");
-        P.use_rest = c.two_phase && c.core_adj == &core.adj && core.rest_built && (rs ? atoi(rs) : 1);
-        if (P.use_rest) P.Rst = view(core.rest);
+        P.Rst = GraphView{};
+        if (c.two_phase && c.rest.ptr && (rs ? atoi(rs) : 1)) P.Rst = c.rest;
         if (P.reduced && c.kind != CG_REACH) {
             P.HB = core.hub_vals.get();
             P.K = core.hub_k;
@@ -1408,6 +1505,7 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
     P.n_src = c.n_src;
     P.two_phase = c.two_phase;
     P.out = c.out;
+    P.out_fmt = c.out_fmt;
     P.p1 = c.two_phase ? c.p1 : nullptr;
     P.V = w.V.get();
     P.M = w.M.get();
@@ -1418,6 +1516,8 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
     P.ctrl = w.ctrl.get();
     P.stats = stats ? st.get() : nullptr;
     P.err = w.err.get();
+    P.err_map = G.sticky_d;
+    P.guard = guard;
     P.max_iters = G.n + 8;
     {
         const char* e = getenv("CG_BITS_BELOW");
@@ -1427,7 +1527,7 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
     }
     CGB_CUDA(cudaMemsetAsync(w.bitmap.get(), 0, w.bitmap.bytes(), s));
     CGB_CUDA(cudaMemsetAsync(w.ctrl.get(), 0, w.ctrl.bytes(), s));
-    CGB_CUDA(cudaMemsetAsync(w.err.get(), 0, 4, s));
+    if (!guard) CGB_CUDA(cudaMemsetAsync(w.err.get(), 0, 4, s));
     if (stats) CGB_CUDA(cudaMemsetAsync(st.get(), 0, st.bytes(), s));
     static const bool tracing = getenv("CG_TRACE") != nullptr;
     DevBuf<unsigned long long> trace, trace_cta;
@@ -1446,7 +1546,6 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
     }
     if (G.packed) launch_kind_b<true>(c.kind, lw, P, G.num_sms, s);
     else launch_kind_b<false>(c.kind, lw, P, G.num_sms, s);
-    CGB_CUDA(cudaMemcpyAsync(err_out, w.err.get(), 4, cudaMemcpyDeviceToHost, s));
     if (tracing) {
         std::vector<unsigned long long> h(5ull * P.trace_cap), hc(2ull * P.trace_cap);
         CGB_CUDA(cudaMemcpyAsync(h.data(), trace.get(), trace.bytes(), cudaMemcpyDeviceToHost, s));
@@ -1492,6 +1591,8 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
             o.scanned_p2 = (int64_t)x[ST_S2];
             o.batch_queries = Q;
             o.row_bytes = (lw == 1 || lw == 2) ? 4 : lw == 33 ? 128 : 64;
+            o.ms_p1 = (float)(x[ST_T1] * 1e-6);
+            o.ms_p2 = (float)(x[ST_T2] * 1e-6);
         }
     }
 }
@@ -1505,21 +1606,20 @@ int batch_width() {
 
 void run_queries_batched(Graph& G, const QueryCall& c, int, cudaStream_t s, std::vector<cg_stats>* stats) {
     const int lw = lane_width(G, c.kind);
-    uint32_t* err = G.bs.err_host();
-    run_batched_lw(G, c, lw, s, stats, err);
-    // f16 SSSP / BFS lanes must know about a lane overflow before the results are trusted: such
-    // a call synchronises once and re-runs with u32 lanes if any candidate reached 2048
+    run_batched_lw(G, c, lw, s, stats, nullptr);
+    // binary16 SSSP / BFS lanes (reading N3) raise ERR_LANE_OVERFLOW when a candidate reaches
+    // 2048; the call is then re-run with u32 lanes.  Without stats the re-run is enqueued
+    // unconditionally and exits at once unless the flag is set (no host synchronisation, so the
+    // call stays asynchronous and capturable); with stats the call synchronises anyway.
     if (lw == 16 && (c.kind == CG_BFS || c.kind == CG_SSSP)) {
-        CGB_CUDA(cudaStreamSynchronize(s));
-        if (*err & ERR_LANE_OVERFLOW) {
-            *err = 0;
-            run_batched_lw(G, c, 32, s, stats, err);
+        if (stats) {
+            uint32_t* err = G.bs.err_host();
+            CGB_CUDA(cudaMemcpyAsync(err, G.bs.err.get(), 4, cudaMemcpyDeviceToHost, s));
+            CGB_CUDA(cudaStreamSynchronize(s));
+            if (*err & ERR_LANE_OVERFLOW) run_batched_lw(G, c, 32, s, stats, nullptr);
+        } else {
+            run_batched_lw(G, c, 32, s, nullptr, G.bs.err.get());
         }
-    }
-    if (stats) {
-        CGB_CUDA(cudaStreamSynchronize(s));
-        CGB_CHECK(!(*err & ERR_SOURCE), CG_EINVAL, "source id >= n");
-        CGB_CHECK(!(*err & ERR_ITERS), CG_EINTERNAL, "iteration bound exceeded");
     }
 }
 

@@ -23,28 +23,43 @@ struct Adj {
     DevBuf<uint2> adjw;
 };
 
+// What a kernel sees of an out-edge structure: row v = edges [ptr[v], end[v]) of adj / adjw,
+// with end == nullptr meaning end[v] = ptr[v+1] (a plain CSR).  The split layout of a Core
+// Graph (below) gives phase 1 the rows [ptr[v], cg_end[v]) and phase 2's first sweep the rows
+// [cg_end[v], ptr[v+1]) of ONE edge array.
 struct GraphView {
     const uint32_t* ptr;
+    const uint32_t* end;
     const uint32_t* adj;
     const uint2* adjw;
 };
 
-inline GraphView view(const Adj& a) { return GraphView{a.ptr.get(), a.adj.get(), a.adjw.get()}; }
+inline GraphView view(const Adj& a) { return GraphView{a.ptr.get(), nullptr, a.adj.get(), a.adjw.get()}; }
 
+// A Core Graph in the split-CSR layout ("the edge lists can
+// be organized to separate critical and non-critical edges so that latter can be easily skipped
+// during the first phase"): ONE copy of G's edges per Core Graph, each row reordered so that
+// its CG edges (canonical order) come first and the others (canonical order) follow:
+//   sadj / sadjw   the reordered edges, row v at G's own offsets [ptr[v], ptr[v+1])
+//   cg_end u32[n]  end of row v's CG part: CG(V, E_c) = rows [ptr[v], cg_end[v])
+// Phase 1 reads the CG rows, phase 2's first sweep the non-CG rows [cg_end[v], ptr[v+1])
+// (reading N7), later phase-2 iterations whole rows.  E_c membership in G's canonical edge
+// order is kept as a bitmap (cg_core_export, persistence, WCC).
 struct Core {
     bool built = false;
     int alg = 0;           // 1 = Algorithm 1 (specialized), 2 = Algorithm 2 (general)
     int connectivity = 0;
-    Adj adj;               // CG(V, E_c) in the engine layout
-    DevBuf<uint8_t> flags; // E_c membership in G's CSR edge order
+    uint32_t m_cg = 0;     // |E_c|
+    DevBuf<uint32_t> sadj; // split rows, packed edge words
+    DevBuf<uint2> sadjw;   // split rows, (dst, w) pairs (wide layout)
+    DevBuf<uint32_t> cg_end;
+    DevBuf<uint32_t> fbits;  // E_c membership bits in G's CSR edge order (bit e of word e/32)
     std::vector<uint32_t> hubs;
     float build_ms = 0.f;
     // NEXT-1 certificates (Theorem 1 P:1321-1371 and its bottleneck analogs): the Identify
     // queries' values kept as rows hub_vals[v][0..2K) = (Q(h_k) on G at v | Q(h_k) on G^R at v)
     DevBuf<uint32_t> hub_vals;
     uint32_t hub_k = 0;
-    Adj rest;              // G minus the CG (phase 2's first sweep, reading N7)
-    bool rest_built = false;
     Adj sym;               // WCC: CG ∪ CG^R (built on the first WCC 2Phase query)
     bool sym_built = false;
 };
@@ -96,9 +111,39 @@ struct Graph {
     bool gsym_built = false;
     Workspace ws;
     BatchSpace bs;
+    // sticky error word of asynchronous calls (ERR_* bits of the engines), in host-mapped pinned
+    // memory: kernels write it through sticky_d, the next API call / cg_graph_status reads sticky_h
+    uint32_t* sticky_h = nullptr;
+    uint32_t* sticky_d = nullptr;
+    // calls on one graph share its workspace: each call's stream waits for the previous call's
+    // work on another stream (event `last`), so calls are serialised per graph across streams
+    cudaEvent_t last = nullptr;
+    cudaStream_t last_stream = nullptr;
+    bool last_valid = false;
+    Graph() = default;
+    Graph(const Graph&) = delete;
+    Graph& operator=(const Graph&) = delete;
+    ~Graph() {
+        if (sticky_h) cudaFreeHost(sticky_h);
+        if (last) cudaEventDestroy(last);
+    }
 };
 
+// engine error bits (both engines); ERR_SOURCE / ERR_ITERS / ERR_NARROW are sticky per graph
+enum : uint32_t { ERR_ITERS = 1u, ERR_SOURCE = 2u, ERR_LANE_OVERFLOW = 4u, ERR_NARROW = 8u };
+
 inline int core_slot(int kind) { return (kind == CG_BFS || kind == CG_WCC) ? CG_REACH : kind; }
+
+// views of a built Core Graph C of G (split layout)
+inline GraphView core_view(const Graph& G, const Core& C) {   // CG(V, E_c): phase 1
+    return GraphView{G.g.ptr.get(), C.cg_end.get(), C.sadj.get(), C.sadjw.get()};
+}
+inline GraphView rest_view(const Graph& G, const Core& C) {   // G minus E_c: phase 2's first sweep
+    return GraphView{C.cg_end.get(), G.g.ptr.get() + 1, C.sadj.get(), C.sadjw.get()};
+}
+inline GraphView split_view(const Graph& G, const Core& C) {  // G with split rows: phase 2
+    return GraphView{G.g.ptr.get(), nullptr, C.sadj.get(), C.sadjw.get()};
+}
 
 // graph_build.cu
 void build_graph(Graph& G, int64_t n, int64_t m, const uint32_t* src, const uint32_t* dst, const uint32_t* w,
@@ -108,14 +153,17 @@ void export_adj(const Graph& G, const Adj& a, int64_t* ptr, uint32_t* idx, uint3
 // engine.cu
 struct QueryCall {
     int kind;
-    Adj* full_adj;         // G (or G^R for backward Identify queries)
-    Adj* core_adj;         // CG (phase 1); ignored when two_phase == 0
+    GraphView full;        // G (or G^R for backward Identify queries); in 2Phase the split rows
+    GraphView core;        // CG (phase 1); ignored when two_phase == 0
+    GraphView rest;        // G minus the CG (phase 2's first sweep, reading N7); ptr null: use full
+    const Core* cg;        // the kind's Core Graph when `core` is it (NEXT-1 certificates), else null
     int two_phase;
     const uint32_t* srcs;  // device
     int32_t n_src;
-    uint32_t* out;         // n_src * n
-    uint32_t* p1;          // nullable
+    void* out;             // n_src rows in out_fmt
+    uint32_t* p1;          // nullable (u32 rows)
     bool want_stats;
+    int out_fmt;           // cg_out_format
 };
 void run_queries(Graph& G, const QueryCall& c, cudaStream_t s, std::vector<cg_stats>* stats);
 
@@ -129,6 +177,7 @@ void build_core_partial(Graph& G, int kind, int32_t K, int policy, const uint32_
 void build_core_from_flags(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs, uint64_t seed,
                            const uint8_t* flags, int connectivity, cudaStream_t s);
 void save_core(Graph& G, int kind, const char* path, cudaStream_t s);
+void export_core_flags(Graph& G, const Core& C, uint8_t* flags, cudaStream_t s);  // u8[m] from the bitmap
 void ensure_wcc_graphs(Graph& G, bool two_phase, cudaStream_t s);  // G ∪ G^R, CG ∪ CG^R for WCC
 void load_core(Graph& G, int kind, const char* path, cudaStream_t s);
 void build_core(Graph& G, int kind, int32_t K, int policy, const uint32_t* hubs, uint64_t seed, int alg,

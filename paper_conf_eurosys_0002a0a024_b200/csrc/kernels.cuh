@@ -95,6 +95,15 @@ template <> struct Op<CG_REACH> {
     __device__ static void edge_fn(uint32_t* p, uint32_t v) { red_max(p, v); }
 };
 
+// the graph's sticky error word lives in host-mapped pinned memory (read by the next API call
+// on the graph, or by cg_graph_status after a stream sync); only thread 0 of the grid writes it
+__device__ __forceinline__ void report_sticky(uint32_t* err_map, uint32_t e) {
+    if (!e || !err_map) return;
+    volatile uint32_t* p = err_map;
+    *p = *p | e;
+    __threadfence_system();
+}
+
 // ------------------------------------------------------------------ grid barrier
 __device__ __forceinline__ void grid_sync(unsigned long long* bar, unsigned long long& epoch) {
     __syncthreads();
@@ -156,7 +165,8 @@ struct EdgeWord<false> {
 };
 
 // Degrees of the 32 vertices of up to CW nonzero bitmap words taken from `nz` (lane = vertex:
-// one coalesced 128 B row-offset read per word; lane 31 fetches the next offset).
+// one coalesced 128 B row-offset read per word; lane 31 fetches the next offset; split rows
+// read their row ends too).
 __device__ __forceinline__ void word_degrees(const GraphView& g, uint32_t n, uint32_t g0, uint32_t& nz, uint32_t lane,
                                              int (&js)[CW], uint32_t (&deg)[CW]) {
     uint32_t p0[CW], p1[CW];
@@ -167,6 +177,20 @@ __device__ __forceinline__ void word_degrees(const GraphView& g, uint32_t n, uin
             js[k] = __ffs(nz) - 1;
             nz &= nz - 1;
         }
+    }
+    if (g.end) {  // split rows: [ptr[v], end[v]) (vertices past n have no row: v < n checked)
+#pragma unroll
+        for (int k = 0; k < CW; ++k) {
+            p0[k] = p1[k] = 0;
+            const uint32_t v = (g0 + js[k]) * 32 + lane;
+            if (js[k] >= 0 && v < n) {
+                p0[k] = __ldg(g.ptr + v);
+                p1[k] = __ldg(g.end + v);
+            }
+        }
+#pragma unroll
+        for (int k = 0; k < CW; ++k) deg[k] = p1[k] - p0[k];
+        return;
     }
 #pragma unroll
     for (int k = 0; k < CW; ++k) {

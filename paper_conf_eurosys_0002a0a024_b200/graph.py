@@ -15,6 +15,7 @@ KINDS = {"sssp": 0, "sswp": 1, "ssnp": 2, "viterbi": 3, "bfs": 4, "reach": 5, "w
 MODES = {"2phase": 0, "full": 1}
 HUB_POLICIES = {"topdeg": 0, "sampled": 1, "given": 2}
 CG_ALGS = {"auto": 0, "specialized": 1, "general": 2, "general_perdir": 3}
+FORMATS = {"u32": 0, "u16": 1, "bits": 2}  # cg_out_format
 
 
 def kind_id(kind) -> int:
@@ -202,27 +203,37 @@ class Graph:
         return flags
 
     # -------------------------------------------------------------- queries
+    def row_shape(self, fmt: str = "u32") -> tuple:
+        """(elements, dtype) of one output row in cg_out_format `fmt`."""
+        if fmt == "u16":
+            return self.n, torch.uint16
+        if fmt == "bits":
+            return (self.n + 31) // 32, torch.uint32
+        return self.n, torch.uint32
+
     def query(self, kind, sources, mode: str = "2phase", out: torch.Tensor | None = None,
-              p1: torch.Tensor | bool | None = None, stats: bool = False):
+              p1: torch.Tensor | bool | None = None, stats: bool = False, fmt: str = "u32"):
         """Evaluate Q(s) for every s in `sources`; returns uint32 [n_src, n] (float32 view for Viterbi).
 
-        p1=True (or a uint32 [n_src, n] tensor) also returns the phase-1 values (2phase only).
-        stats=True returns per-query counters (synchronises)."""
+        fmt: "u32" (default), "u16" (uint16 rows, 0xFFFFFFFF as 0xFFFF) or "bits" (REACH: bit-packed
+        uint32 rows) — cg_out_format.  p1=True (or a uint32 [n_src, n] tensor) also returns the
+        phase-1 values (2phase only).  stats=True returns per-query counters (synchronises)."""
         k = kind_id(kind)
         if k == KINDS["wcc"] and sources is None:  # whole-graph query: one row of labels
             sources = [0]
         src = _u32(sources, self.device).reshape(-1)
         ns = src.numel()
         if out is None:
-            out = torch.empty((ns, self.n), dtype=torch.uint32, device=self.device)
+            cols, dt = self.row_shape(fmt)
+            out = torch.empty((ns, cols), dtype=dt, device=self.device)
         if p1 is True:
             p1 = torch.empty((ns, self.n), dtype=torch.uint32, device=self.device)
         st = (_lib.Stats * max(ns, 1))() if stats else None
         with torch.cuda.device(self.device):
-            _lib.call("cg_query_ex", self._h, k, _ptr(src), ns, MODES[mode], _ptr(out),
+            _lib.call("cg_query_fmt", self._h, k, _ptr(src), ns, MODES[mode], FORMATS[fmt], _ptr(out),
                       _ptr(p1) if isinstance(p1, torch.Tensor) else None,
                       ctypes.cast(st, ctypes.c_void_p) if st is not None else None, _stream(self.device))
-        res = out.view(torch.float32) if k == KINDS["viterbi"] else out
+        res = out.view(torch.float32) if (k == KINDS["viterbi"] and fmt == "u32") else out
         extra = []
         if isinstance(p1, torch.Tensor):
             extra.append(p1.view(torch.float32) if k == KINDS["viterbi"] else p1)
@@ -231,18 +242,25 @@ class Graph:
         return (res, *extra) if extra else res
 
     def query_host(self, kind, sources, mode: str = "2phase", out: torch.Tensor | None = None,
-                   batch: int = 0) -> torch.Tensor:
-        """cg_query_host: host sources in, host (pinned) values out, copies overlapped with compute."""
+                   batch: int = 0, fmt: str = "u32") -> torch.Tensor:
+        """cg_query_host_fmt: host sources in, host (pinned) values out in `fmt`, copies overlapped
+        with compute."""
         k = kind_id(kind)
         src = sources if isinstance(sources, torch.Tensor) else torch.as_tensor(sources)
         src = src.to(torch.int64).to(torch.uint32).contiguous().cpu()
         ns = src.numel()
         if out is None:
-            out = torch.empty((ns, self.n), dtype=torch.uint32, pin_memory=True)
+            cols, dt = self.row_shape(fmt)
+            out = torch.empty((ns, cols), dtype=dt, pin_memory=True)
         with torch.cuda.device(self.device):
-            _lib.call("cg_query_host", self._h, k, _ptr(src), ns, MODES[mode], _ptr(out), int(batch),
-                      _stream(self.device))
-        return out.view(torch.float32) if k == KINDS["viterbi"] else out
+            _lib.call("cg_query_host_fmt", self._h, k, _ptr(src), ns, MODES[mode], FORMATS[fmt], _ptr(out),
+                      int(batch), _stream(self.device))
+        return out.view(torch.float32) if (k == KINDS["viterbi"] and fmt == "u32") else out
+
+    def status(self) -> None:
+        """cg_graph_status: synchronise and raise the graph's pending sticky device error, if any."""
+        with torch.cuda.device(self.device):
+            _lib.call("cg_graph_status", self._h, _stream(self.device))
 
 
 def kernel_launches() -> int:

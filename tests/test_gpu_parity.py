@@ -145,7 +145,8 @@ def test_wide_weights_use_u32_lanes():
 
 
 def test_star_hub_chunks():
-    """A hub with 10^6 out-edges exercises the multi-CTA chunk tier (rows >= kBigThreshold)."""
+    """A hub with 10^6 out-edges: its row is split over many warps and CTAs by the edge-balanced
+    S2 (a window row longer than any warp's share, dynamic tail tiles)."""
     leaves = 1_000_000
     n = leaves + 2
     src = np.concatenate([np.zeros(leaves, np.uint32), np.arange(1, 2001, dtype=np.uint32)])
@@ -255,22 +256,20 @@ def test_alg_options_match_oracle():
     assert np.array_equal(g.core_flags("reach").cpu().numpy(), oracle.cg_alg2(og, ogr, hubs, connectivity=True))
 
 
-@pytest.mark.parametrize("dense_div", ["0", "8", "4294967295"])
-def test_dense_and_sparse_iterations(dense_div, monkeypatch):
-    """Force every iteration sparse (list + balanced split), the default mix, or every
-    iteration dense (TMA-streamed edge slices): all must give the oracle's values.  A graph
-    large enough for multi-chunk slices, skipped inactive hub rows and many warps per row."""
-    monkeypatch.setenv("CG_DENSE_DIV", dense_div)
+def test_rmat18_all_kinds_many_tiles():
+    """A mid-size graph (2^18 vertices, 4 M edges): many S1 rounds per CTA, multi-window hub
+    rows shared by several warps and CTAs, dense and sparse frontiers in both phases — every kind
+    in both modes against the oracle."""
     n, m = 1 << 18, 16 << 18
     src, dst, w = gen.rmat(n, m, w_max=19, seed=13)
     g, og = both(n, src, dst, w)
     sources = np.concatenate([[0], gen.sample_sources(n, src, dst, 5, seed=2)]).astype(np.uint32)
-    for kind in ("sssp", "viterbi", "bfs", "sswp"):
+    for kind in KINDS:
         g.build(kind, K=20)
         for mode in ("full", "2phase"):
             out = to_np(g.query(kind, to_dev(sources), mode=mode))
             for i, s in enumerate(sources):
-                assert_values_equal(out[i], oracle.query(kind, og, int(s)), kind, f"{kind}/{mode}/div={dense_div}/s={s}")
+                assert_values_equal(out[i], oracle.query(kind, og, int(s)), kind, f"{kind}/{mode}/s={s}")
 
 
 @pytest.mark.parametrize("engine", ["single", "u32", "packed"])
@@ -418,8 +417,15 @@ def test_partial_builds_merge_to_full_core_graph(kind):
         f = g.build_partial(kind, K=20, hub_range=(b, e))
         merged = f.clone() if merged is None else torch.maximum(merged, f)
     info = g.build_from_flags(kind, merged, K=20)
-    assert np.array_equal(g.core_flags(kind).cpu().numpy(), ref_flags)
-    assert info["m_cg"] == ref["m_cg"] and info["hubs"] == ref["hubs"]
+    ogr = oracle.transpose(og)
+    exp = oracle.cg_alg1(kind, og, ogr, np.array(ref["hubs"], np.uint32), connectivity=True)
+    assert np.array_equal(ref_flags, exp)  # the single-call build is the oracle's Algorithm 1 CG
+    assert np.array_equal(g.core_flags(kind).cpu().numpy(), exp)  # ... and so is the merged one
+    assert info["m_cg"] == ref["m_cg"] == int(exp.sum()) and info["hubs"] == ref["hubs"]
+    # the shards' raw flags are the oracle's Alg 1 marks of their hubs (no connectivity edges)
+    f0 = g.build_partial(kind, K=20, hub_range=(0, 7)).cpu().numpy()
+    assert np.array_equal(f0, oracle.cg_alg1(kind, og, ogr, np.array(ref["hubs"][:7], np.uint32),
+                                             connectivity=False))
     sources = gen.sample_sources(n, src, dst, 9, seed=2)
     out = to_np(g.query(kind, to_dev(sources), mode="2phase"))
     for i, s in enumerate(sources):
@@ -444,7 +450,12 @@ def test_core_graph_save_load(tmp_path):
         g2 = Graph(n, to_dev(src), to_dev(dst), to_dev(w))
         info2 = g2.load_core(kind, path)
         assert info2["m_cg"] == info["m_cg"] and info2["hubs"] == info["hubs"]
-        assert np.array_equal(g2.core_flags(kind).cpu().numpy(), g.core_flags(kind).cpu().numpy())
+        ogr = oracle.transpose(og)
+        hubs = np.array(info["hubs"], np.uint32)
+        exp = (oracle.cg_alg1(kind, og, ogr, hubs) if kind == "sssp"
+               else oracle.cg_alg2(og, ogr, hubs, per_direction=True))  # the kind's CG (reading Q9')
+        assert np.array_equal(g2.core_flags(kind).cpu().numpy(), exp)  # loaded == oracle CG
+        assert np.array_equal(g.core_flags(kind).cpu().numpy(), exp)
         out = to_np(g2.query(kind, to_dev(sources), mode="2phase"))
         for i, s in enumerate(sources):
             assert_values_equal(out[i], oracle.query(kind, og, int(s)), kind, f"loaded {kind} s={s}")

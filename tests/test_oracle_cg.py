@@ -118,12 +118,15 @@ def test_alg2_worked_example():
     assert list(flags) == [int(x) for x in gd["flags"][0]]
 
 
-def _alg2_levelsync(g, gr, hubs):
+def _alg2_levelsync(g, gr, hubs, per_direction=False):
     """Independent formulation of Alg 2: level-synchronous traversal where each newly
     labeled vertex's discovering edge is the one with minimum (rank of parent in FIFO
-    order, position in the parent's adjacency), and the next level is ordered by that key."""
+    order, position in the parent's adjacency), and the next level is ordered by that key.
+    per_direction: one label array for the forward traversals and one for the backward ones
+    (reading Q9')."""
     n = g.n
-    qid = np.zeros(n, dtype=np.int64)
+    qids = {False: np.zeros(n, dtype=np.int64)}
+    qids[True] = np.zeros(n, dtype=np.int64) if per_direction else qids[False]
     flags = np.zeros(g.m, dtype=np.uint8)
 
     def g_edge(u, v):  # position of G edge u->v
@@ -135,6 +138,7 @@ def _alg2_levelsync(g, gr, hubs):
     for k, h in enumerate(hubs):
         lab = k + 1
         for graph, rev in ((g, False), (gr, True)):
+            qid = qids[rev]
             level = [int(h)]
             while level:
                 win = {}
@@ -169,6 +173,39 @@ def test_alg2_equals_levelsync_formulation(seed):
     gr = oracle.transpose(g)
     hubs = oracle.hubs_topdeg(g, gr, min(5, n))
     assert np.array_equal(oracle.cg_alg2(g, gr, hubs), _alg2_levelsync(g, gr, hubs))
+    # the per-direction variant (reading Q9', the default general CG of BFS / REACH / WCC)
+    assert np.array_equal(oracle.cg_alg2(g, gr, hubs, per_direction=True),
+                          _alg2_levelsync(g, gr, hubs, per_direction=True))
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_alg2_per_direction_is_union_of_directions(seed):
+    """With one Qid per direction, the forward traversals never see the backward labels and vice
+    versa, so the CG is the union of Alg 2 run forward-only on G and forward-only on G^R (its
+    edges reversed back into G, Alg 2 l.9): a mistake such as the backward traversal reusing
+    the forward labels, or not reversing its edges, breaks this identity."""
+    if seed < 2:
+        rng = np.random.default_rng(100 + seed)
+        n = int(rng.integers(3, 60))
+        src, dst, w = random_multigraph(rng, n, 5 * n)
+    else:
+        n, src, dst, w = rmat_small(9, 8, 30 + seed)
+    g = oracle.canonical_csr(n, src, dst, w)
+    gr = oracle.transpose(g)
+    hubs = oracle.hubs_topdeg(g, gr, min(6, n))
+    empty = oracle.CSR(n, np.zeros(n + 1, np.int64), np.zeros(0, np.uint32), np.zeros(0, np.uint32))
+    fwd = oracle.cg_alg2(g, empty, hubs)                 # forward traversals only, on G
+    bwd_r = oracle.cg_alg2(gr, empty, hubs)              # forward-only on G^R: flags in G^R's order
+    bwd = np.zeros(g.m, np.uint8)                        # G^R edge (v -> u) is G edge (u -> v)
+    for v in range(n):
+        for i in range(int(gr.ptr[v]), int(gr.ptr[v + 1])):
+            if bwd_r[i]:
+                u = int(gr.col[i])
+                lo, hi = int(g.ptr[u]), int(g.ptr[u + 1])
+                bwd[lo + int(np.searchsorted(g.col[lo:hi], v))] = 1
+    union = np.maximum(fwd, bwd)
+    per_dir = oracle.cg_alg2(g, gr, hubs, per_direction=True)
+    assert np.array_equal(per_dir, union)
 
 
 @pytest.mark.parametrize("seed", [3, 4])

@@ -205,3 +205,21 @@ def test_wcc_oracle_pins(seed):
     rows = np.repeat(np.arange(n), np.diff(g.ptr))
     assert np.array_equal(lab[rows], lab[g.col])
     assert np.array_equal(oracle.query("wcc", g, 0), lab)
+
+
+@pytest.mark.parametrize("kind", KINDS)
+def test_query_batch_equals_single_queries(kind):
+    """or_query_batch (the OpenMP driver the full-size parity tests and the CPU baseline use)
+    returns, row by row, exactly or_query of each source — any thread count, repeated and
+    out-of-order sources included; or_query itself is pinned above (brute force, scipy,
+    threshold reachability, closed forms)."""
+    n, src, dst, w = rmat_small(10, 8, 91)
+    g = oracle.canonical_csr(n, src, dst, w)
+    rng = np.random.default_rng(5)
+    sources = np.concatenate([rng.integers(0, n, 13), [7, 7, 0, n - 1]]).astype(np.uint32)
+    for threads in (1, 3, 8):
+        out = oracle.query_batch(kind, g, sources, nthreads=threads)
+        assert out.shape == (sources.size, n)
+        for i, s in enumerate(sources):
+            assert np.array_equal(out[i], oracle.query(kind, g, int(s))), (kind, threads, i)
+    assert oracle.query_batch(kind, g, np.zeros(0, np.uint32)).shape == (0, n)
