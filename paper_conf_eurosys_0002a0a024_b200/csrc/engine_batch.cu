@@ -161,12 +161,13 @@ struct Lanes16 {
     static constexpr uint32_t INF16 = 0x7c00u, LIMIT = 0x68006800u;  // +inf; 2048.0 in both lanes
     static constexpr uint32_t INIT16 = MAXK ? 0u : INF16, SRC16 = MAXK ? INF16 : 0u;
     __device__ static uint32_t init_word() { return INIT16 * 0x10001u; }
-    // lane j as a u32: values are integers in [0, 2048) (or +inf), so the binary16 pattern
-    // decodes with integer ops — significand with its hidden bit, shifted by 25 - biased
-    // exponent (0 -> 0 falls out of the shift) — instead of two quarter-rate conversions
+    // lane j as a u32: values are integers in [0, 2048] (or +inf), so the binary16 pattern
+    // decodes with integer ops — significand with its hidden bit, times 2, shifted right by
+    // 26 - biased exponent (0 -> 0 falls out of the shift; exponent 26 is 2048) — instead of
+    // two quarter-rate conversions
     __device__ static uint32_t decode(uint32_t x, uint32_t j) {
         const uint32_t h = (x >> (16 * j)) & 0xffffu;
-        const uint32_t k = ((h & 0x3ffu) | 0x400u) >> min(25u - (h >> 10), 31u);
+        const uint32_t k = (((h & 0x3ffu) | 0x400u) << 1) >> min(26u - (h >> 10), 31u);
         return h == INF16 ? 0xffffffffu : k;
     }
     __device__ static uint32_t bits2(uint32_t m) { return ((m >> 15) & 1u) | ((m >> 30) & 2u); }  // 0xffff lanes -> 2 bits
