@@ -1121,8 +1121,8 @@ __device__ void transpose_narrow(const BParams& P, int q0, int nq, uint32_t* xs)
     const uint32_t gw = blockIdx.x * BW + (threadIdx.x >> 5);
     const uint32_t NW = gridDim.x * BW;
     const uint32_t T = (P.n + 31) / 32;  // tiles
-    if constexpr (L::QPW == 32) {  // bit lanes: CG_OUT_BITS (the host admits REACH's bit lanes only)
-        if (P.out_fmt != CG_OUT_BITS) return;
+    if constexpr (L::QPW == 32) {  // bit lanes: CG_OUT_BITS (the host admits REACH only)
+      if (P.out_fmt == CG_OUT_BITS) {
         uint32_t* dst = static_cast<uint32_t*>(P.out);
         for (uint32_t tile = gw; tile < T; tile += NW) {
             const uint32_t v = tile * 32 + lane;
@@ -1135,6 +1135,7 @@ __device__ void transpose_narrow(const BParams& P, int q0, int nq, uint32_t* xs)
             if ((int)lane < nq) __stcs(dst + (size_t)(q0 + lane) * T + tile, mine);
         }
         return;
+      }
     }
     if (P.out_fmt != CG_OUT_U16) return;
     uint16_t* dst = static_cast<uint16_t*>(P.out);
