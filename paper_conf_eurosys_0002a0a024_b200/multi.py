@@ -63,3 +63,44 @@ def build_sharded(graph, kind, K: int = 20, rank: int = 0, world: int = 1, group
     flags = graph.build_partial(kind, K=K, hub_range=(b, e), **kw)
     merge_flags(flags, group)
     return graph.build_from_flags(kind, flags, K=K, **kw)
+
+
+class GatherRing:
+    """Double-buffered result gather to rank 0 (the path's single exchange step).
+
+    Step i writes its value rows into slot i % slots and starts an asynchronous gather of them;
+    before step i + slots rewrites that slot, ``acquire`` waits for step i's gather (a stream
+    wait, no host sync), so a gather never reads a block that a later step is overwriting.
+    Rank 0 gathers each slot into that slot's own root buffers.  Blocks travel as bytes, so any
+    dtype works (uint16 / bit-packed narrow rows, uint32 rows)."""
+
+    def __init__(self, rank: int, world: int, slots: int = 2):
+        self.rank, self.world, self.slots = rank, world, slots
+        self.works = [[] for _ in range(slots)]
+        self.roots = [{} for _ in range(slots)]
+
+    def acquire(self, slot: int) -> None:
+        for w in self.works[slot]:
+            w.wait()
+        self.works[slot] = []
+
+    def submit(self, slot: int, key, block: torch.Tensor) -> None:
+        if self.world == 1:
+            return
+        raw = block.view(torch.uint8) if block.dtype != torch.uint8 else block
+        bufs = None
+        if self.rank == 0:
+            bufs = self.roots[slot].get(key)
+            if bufs is None or bufs[0].shape != raw.shape:
+                bufs = [torch.empty_like(raw) for _ in range(self.world)]
+                self.roots[slot][key] = bufs
+        _, work = gather_rows(raw, self.rank, self.world, bufs, async_op=True)
+        self.works[slot].append(work)
+
+    def gathered(self, slot: int, key):
+        """Rank 0: the world's blocks of `key` in `slot` (valid after acquire / drain)."""
+        return self.roots[slot].get(key)
+
+    def drain(self) -> None:
+        for s in range(self.slots):
+            self.acquire(s)

@@ -35,3 +35,26 @@ def test_reference_arm_other_ranks_exit_quietly():
                         "--steps", "1", "--warmup", "0"], capture_output=True, text=True, timeout=300, cwd=ROOT,
                        env=env)
     assert r.returncode == 0 and r.stdout.strip() == ""
+
+
+def test_launch_plan_relaunch_and_mismatch():
+    """`--gpus N` without a torchrun environment re-launches under torch.distributed.run with N
+    ranks on 127.0.0.1; a torchrun environment whose WORLD_SIZE differs from --gpus is refused."""
+    sys.path.insert(0, ROOT)
+    import bench
+    assert bench.launch_plan(1, {}) == "run"
+    assert bench.launch_plan(8, {}) == "relaunch"
+    assert bench.launch_plan(4, {"WORLD_SIZE": "4"}) == "run"
+    msg = bench.launch_plan(4, {"WORLD_SIZE": "2"})
+    assert msg not in ("run", "relaunch") and "WORLD_SIZE=2" in msg
+    cmd = bench.torchrun_cmd(["--gpus", "8", "--steps", "3"], 8, 29511)
+    assert cmd[1:4] == ["-m", "torch.distributed.run", "--nnodes=1"]
+    assert "--nproc-per-node=8" in cmd and "--master-addr=127.0.0.1" in cmd and "--master-port=29511" in cmd
+    assert cmd[-4:] == ["--gpus", "8", "--steps", "3"] and cmd[-5].endswith("bench.py")
+
+
+def test_world_size_mismatch_exits_before_any_gpu_work():
+    env = dict(os.environ, RANK="0", WORLD_SIZE="2", LOCAL_RANK="0")
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "4", "--steps", "1"],
+                       capture_output=True, text=True, timeout=300, cwd=ROOT, env=env)
+    assert r.returncode == 2 and "WORLD_SIZE=2" in r.stderr and r.stdout.strip() == ""

@@ -112,3 +112,40 @@ def test_sharded_core_graph_merge_world2(tmp_path):
     gr = oracle.transpose(g)
     exp = oracle.cg_alg1("sswp", g, gr, oracle.hubs_topdeg(g, gr, K), connectivity=False)
     assert np.array_equal(np.load(out), exp)
+
+
+def _ring_worker(rank, world, port, out_path):
+    sys.path.insert(0, ROOT)
+    from paper_conf_eurosys_0002a0a024_b200 import multi
+
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    ring = multi.GatherRing(rank, world, slots=2)
+    blocks = [torch.zeros((3, 5), dtype=torch.int16) for _ in range(2)]  # the two output slots
+    seen = []
+    for i in range(7):
+        slot = i % 2
+        ring.acquire(slot)  # step i-2's gather of this slot has finished
+        if rank == 0 and i >= 2:  # ... so the root buffers hold step i-2's rows, whole
+            seen.append([int(b.view(torch.int16)[0, 0]) for b in ring.gathered(slot, "k")])
+        blocks[slot].fill_(100 * i + rank)  # step i overwrites its slot
+        ring.submit(slot, "k", blocks[slot])
+    ring.drain()
+    if rank == 0:
+        for i in (5, 6):
+            seen.append([int(b.view(torch.int16)[0, 0]) for b in ring.gathered(i % 2, "k")])
+        np.save(out_path, np.array(seen))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_gather_ring_slot_reuse_world2(tmp_path):
+    """The bench's double-buffered gather (multi.GatherRing): a slot is rewritten only after the
+    gather that read it finished, and rank 0's per-slot root buffers hold exactly the step that
+    was gathered into them (no write-after-read race between step i's gather and step i+2)."""
+    out = str(tmp_path / "seen.npy")
+    mp.spawn(_ring_worker, args=(2, _free_port(), out), nprocs=2, join=True)
+    seen = np.load(out)
+    exp = np.array([[100 * i, 100 * i + 1] for i in range(7)])
+    assert np.array_equal(seen, exp)
