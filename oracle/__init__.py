@@ -17,6 +17,8 @@ Parity status:
   cg_alg1                     pinned (Table 2 / Fig 4 golden; hub-query preservation property)
   cg_alg2                     pinned (hand-worked golden; reachability preservation property)
   two_phase / full_bsp        pinned (== query on every vertex; complete-CG exactness; p1 <= final)
+  certified (O7)              pinned (certified => precise on every vertex; hubs reached in phase 1
+                              are certified by Theorem 1 (a); closed forms on a path graph)
 """
 from __future__ import annotations
 
@@ -77,6 +79,7 @@ def _load():
         "or_2phase": (None, [c_int, i64, P, P, P, P, P, P, u32, P, P, ctypes.POINTER(_Stats)]),
         "or_full_bsp": (None, [c_int, i64, P, P, P, u32, P, ctypes.POINTER(_Stats)]),
         "or_wcc": (None, [i64, P, P, P]),
+        "or_certified": (None, [c_int, i64, u32, P, i32, P, P, P]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -246,3 +249,22 @@ def cg_for_kind(kind, g: CSR, gr: CSR, hubs) -> np.ndarray:
 def as_float(vals: np.ndarray) -> np.ndarray:
     """Viterbi value words -> float32 view."""
     return np.ascontiguousarray(vals, dtype=np.uint32).view(np.float32)
+
+
+def hub_values(kind, g: CSR, gr: CSR, hubs):
+    """The Identify queries' values (Alg 1 l.4-5): (hf, hb) with hf[k] = Q(h_k) on G ("d(h, .)")
+    and hb[k] = Q(h_k) on G^R ("d(., h)"), each [K, n] uint32."""
+    hf = np.stack([query(kind, g, int(h)) for h in hubs]) if len(hubs) else np.zeros((0, g.n), np.uint32)
+    hb = np.stack([query(kind, gr, int(h)) for h in hubs]) if len(hubs) else np.zeros((0, g.n), np.uint32)
+    return np.ascontiguousarray(hf, dtype=np.uint32), np.ascontiguousarray(hb, dtype=np.uint32)
+
+
+def certified(kind, s: int, p1: np.ndarray, hf: np.ndarray, hb: np.ndarray) -> np.ndarray:
+    """O7 (NEXT-1): u8[n], 1 where Theorem 1 or its SSWP / SSNP bottleneck analog
+    (or REACH's lattice top) proves the phase-1 value p1(v) precise (see oracle.c)."""
+    p1 = np.ascontiguousarray(p1, dtype=np.uint32)
+    n = p1.size
+    out = np.zeros(max(n, 1), dtype=np.uint8)
+    _load().or_certified(_kind(kind), n, int(s), _p(_nz(p1)), int(hf.shape[0]), _p(_nz(hf.reshape(-1))),
+                         _p(_nz(hb.reshape(-1))), _p(out))
+    return out[:n].copy()

@@ -33,6 +33,9 @@
  *    sequential BSP order (readings Q1-Q5).
  *  - or_wcc: weakly connected components (NEXT-3, Table 6 WCC row): the
  *    minimum vertex id of each weak component, by union-find.
+ *  - or_certified: O7, the precision certificates of the Reduced(E)
+ *    optimization (NEXT-1): Theorem 1 for SSSP / BFS, its
+ *    bottleneck analogs for SSWP / SSNP, the lattice top for REACH.
  *
  * Value words: every kind stores a 32-bit word per vertex; Viterbi stores
  * the IEEE-754 binary32 bit pattern (reading Q13: f32, RN division).
@@ -614,4 +617,47 @@ void or_wcc(int64_t n, const int64_t* ptr, const uint32_t* col, uint32_t* out) {
         }
     for (int64_t v = 0; v < n; ++v) out[v] = (uint32_t)uf_find(par, v);
     free(par);
+}
+
+/* ---------------------------------------------------------------- O7 (NEXT-1)
+ * Which phase-1 values are PROVEN precise.  p1 = Val(s, v) on the CG after phase 1;
+ * hf[k*n + v] = Q(h_k) on G at v (forward Identify query, "d(h, v).G"), hb[k*n + v] = Q(h_k) on
+ * G^R at v ("d(v, h).G"), for the K hubs the CG was built from.  out[v] = 1 iff v is reached in
+ * phase 1 and some hub certifies it:
+ *   SSSP / BFS, Theorem 1:
+ *     (a) p1(v) == d(s,h) - d(v,h)      (b) p1(v) == d(h,v) - d(h,s)
+ *     (the right-hand sides are lower bounds of d(s,v) by the triangle inequality, P:1338-1366;
+ *     p1 is an upper bound because CG is a subgraph of G; both d's must be finite)
+ *   SSWP (max of path minima; p1 <= W(s,v) because CG is a subgraph): the bottleneck triangle
+ *     W(s,h) >= min(W(s,v), W(v,h)) gives, when W(v,h) > W(s,h), the upper bound W(s,v) <= W(s,h);
+ *     likewise W(h,v) >= min(W(h,s), W(s,v)) gives W(s,v) <= W(h,v) when W(h,s) > W(h,v).
+ *     (a) W(v,h) > W(s,h) and p1(v) == W(s,h)     (b) W(h,s) > W(h,v) and p1(v) == W(h,v)
+ *   SSNP (min of path maxima; p1 >= N(s,v)): mirror images,
+ *     (a) N(v,h) < N(s,h) and p1(v) == N(s,h)     (b) N(h,s) < N(h,v) and p1(v) == N(h,v)
+ *   REACH: p1(v) == 1 (the lattice top, final by definition).
+ * Viterbi has no exact certificate here (its triangle bound needs a rounded division). */
+void or_certified(int kind, int64_t n, uint32_t s, const uint32_t* p1, int32_t K, const uint32_t* hf,
+                  const uint32_t* hb, uint8_t* out) {
+    const uint32_t INF = 0xFFFFFFFFu;
+    for (int64_t v = 0; v < n; ++v) {
+        out[v] = 0;
+        const uint32_t p = p1[v];
+        if (p == or_init_val(kind)) continue;                        /* not reached in phase 1 */
+        if (kind == K_REACH) { out[v] = p == 1u; continue; }
+        for (int32_t k = 0; k < K && !out[v]; ++k) {
+            const uint32_t* f = hf + (size_t)k * (size_t)n;         /* d(h, .) */
+            const uint32_t* b = hb + (size_t)k * (size_t)n;         /* d(., h) */
+            const uint32_t d_sh = b[s], d_vh = b[v], d_hv = f[v], d_hs = f[s];
+            if (kind == K_SSSP || kind == K_BFS) {
+                if (d_sh != INF && d_vh != INF && d_sh >= d_vh && p == d_sh - d_vh) out[v] = 1;   /* (a) */
+                if (d_hv != INF && d_hs != INF && d_hv >= d_hs && p == d_hv - d_hs) out[v] = 1;   /* (b) */
+            } else if (kind == K_SSWP) {
+                if (d_vh > d_sh && p == d_sh) out[v] = 1;                                        /* (a) */
+                if (d_hs > d_hv && p == d_hv) out[v] = 1;                                        /* (b) */
+            } else if (kind == K_SSNP) {
+                if (d_vh < d_sh && p == d_sh) out[v] = 1;                                        /* (a) */
+                if (d_hs < d_hv && p == d_hv) out[v] = 1;                                        /* (b) */
+            }
+        }
+    }
 }
