@@ -380,10 +380,11 @@ def run_c1_single(ctx):
     cfg = gen.CONFIGS["c1"]
     g, _ = build_graph(cfg, ctx.dev)
     g.build("sssp", K=20)
-    src = torch.zeros(1, dtype=torch.uint32, device=ctx.dev)
+    v0 = gen.generator_vertex(cfg, 0)  # reading N10: the generator's vertex 0 (the top hub)
+    src = torch.full((1,), v0, dtype=torch.int64).to(torch.uint32).to(ctx.dev)
     out = torch.empty((1, cfg.n), dtype=torch.uint32, device=ctx.dev)
     flush = torch.empty(64 << 20, dtype=torch.int32, device=ctx.dev)
-    res = {"workload": cfg.name, "query": "SSSP from vertex 0", "K_hubs": 20,
+    res = {"workload": cfg.name, "query": f"SSSP from the generator's vertex 0 (id {v0}, reading N10)", "K_hubs": 20,
            "l2": "flushed before every timed query (256 MB write outside the events)"}
     steps = 200
     for mode in ("2phase", "full"):

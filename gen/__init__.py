@@ -81,6 +81,14 @@ def rmat(n: int, m: int, abcd=(0.57, 0.19, 0.19, 0.05), w_max: int = 64, seed: i
     return src, dst, w
 
 
+def generator_vertex(cfg, x: int = 0) -> int:
+    """Vertex x of the R-MAT generator (before the vertex-id permutation) in the permuted ids of
+    `cfg`'s graph.  BASELINE configs[0] queries "vertex 0": in an unpermuted Graph500 R-MAT that is
+    the a-quadrant corner, the highest-degree vertex; after the permutation it is
+    gen_permute(0) (reading N10).  Id 0 of the permuted graph is an isolated vertex."""
+    return int(_load().gen_permute(x, cfg.n, cfg.seed))
+
+
 def log_weight_max(n: int) -> int:
     """Paper's weight range upper end log(n)+1, read as floor(log2 n)+1."""
     return int(math.floor(math.log2(max(n, 2)))) + 1

@@ -1190,7 +1190,7 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
     // thread 0's bookkeeping lives in shared memory (not registers live across the loop):
     // sticky errors of this launch, and the pass's start / phase-switch times (stats)
     __shared__ uint32_t sm_err;
-    __shared__ unsigned long long sm_t[2];
+    __shared__ unsigned long long sm_t[4];  // pass start, phase switch, phase 2 start, values written
     if (threadIdx.x == 0) sm_err = 0u;
 
     // kernel-level trace marks (tid 0): [cap-1] = {entry, seeds done, loop done, exit} of batch 0
@@ -1198,7 +1198,7 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
     if (kt) kt[0] = global_ns();
     for (int q0 = 0; q0 < P.n_src; q0 += Q) {
         const int nq = min(Q, P.n_src - q0);
-        if (P.stats && tid == 0) sm_t[0] = sm_t[1] = global_ns();
+        if (P.stats && tid == 0) sm_t[0] = sm_t[1] = sm_t[2] = global_ns();
         // Alg 3 l.4, l.6 for every query of the batch; masks cleared
         if constexpr (RW % 4 == 0 && !InitOf<L>::ALL_ACTIVE) {  // 16 B stores
             const uint32_t iw = L::init_word();
@@ -1302,6 +1302,7 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
                 n_edges = n_upd = n_read = 0;
                 iters = 0;
                 if (phase == 1) {
+                    if (P.stats && tid == 0) sm_t[1] = global_ns();  // (the counters' own passes excluded)
                     if (P.p1) transpose_out<L>(P, P.p1, q0, nq, xs, vs);
                     if (P.stats) {  // impacted per query (Alg 3 l.15); the thread's query q is fixed
                         const uint32_t q = (uint32_t)(tid % Q);
@@ -1313,7 +1314,7 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
                     }
                     // the p1 / impacted reads must finish before phase 2 updates V
                     if (P.p1 || P.stats) grid_sync(P.ctrl, epoch);
-                    if (P.stats && tid == 0) sm_t[1] = global_ns();
+                    if (P.stats && tid == 0) sm_t[2] = global_ns();
                     phase = 2;
                     if (P.reduced) pull = true;   // Reduced(E): pull into uncertified vertices
                     else predicate = true;        // Active <- impacted vertices (l.15)
@@ -1356,6 +1357,8 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
             else transpose_narrow<L>(P, q0, nq, xs);
         }
         if (P.stats) {  // reached / precise per query (the thread's query q is fixed)
+            grid_sync(P.ctrl, epoch);  // every CTA's values written: the phase-2 end time
+            if (tid == 0) sm_t[3] = global_ns();
             const uint32_t q = (uint32_t)(tid % Q);
             const uint32_t sb = ((int)q < nq && P.srcs) ? __ldg(P.srcs + q0 + q) : 0xffffffffu;
             const uint32_t init = L::decode(L::init_word(), 0);
@@ -1373,10 +1376,9 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
         }
         grid_sync(P.ctrl, epoch);  // V / M / bitmap are reused by the next batch
         if (P.stats && tid == 0) {  // device time of this pass's phases, for each of its queries
-            const unsigned long long t_end = global_ns();
             for (int b = 0; b < nq; ++b) {
                 atomicAdd(P.stats + (size_t)(q0 + b) * NSTAT + ST_T1, sm_t[1] - sm_t[0]);
-                atomicAdd(P.stats + (size_t)(q0 + b) * NSTAT + ST_T2, t_end - sm_t[1]);
+                atomicAdd(P.stats + (size_t)(q0 + b) * NSTAT + ST_T2, sm_t[3] - sm_t[2]);
             }
         }
     }

@@ -51,3 +51,17 @@ def test_sample_sources():
     src = gen.sample_sources(n, s, d, 10, seed=42)
     assert src.size == 10 and np.all(np.isin(src, s[s != d]))
     assert np.array_equal(src, gen.sample_sources(n, s, d, 10, seed=42))
+
+
+def test_generator_vertex_zero_is_the_top_hub():
+    """Reading N10: configs[0]'s "vertex 0" is the R-MAT generator's vertex 0, which the Feistel
+    permutation moves; it is the highest-degree vertex of the C1 graph, while id 0 is isolated."""
+    c = gen.CONFIGS["c1"]
+    s, d, _ = c.edges()
+    v0 = gen.generator_vertex(c, 0)
+    keep = s != d
+    deg = np.bincount(s[keep], minlength=c.n) + np.bincount(d[keep], minlength=c.n)
+    assert deg.argmax() == v0 and deg[0] == 0
+    u, v, _ = gen.rmat(c.n, 1000, c.abcd, c.w_max, c.seed, permute=False)
+    up, vp, _ = gen.rmat(c.n, 1000, c.abcd, c.w_max, c.seed, permute=True)
+    assert all(gen.generator_vertex(c, int(a)) == int(b) for a, b in zip(u[:50], up[:50]))

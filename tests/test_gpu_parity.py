@@ -84,10 +84,12 @@ def test_queries_small_random(seed):
 
 
 def test_queries_rmat16_config1():
-    """configs[0]: RMAT scale-16 ef16, w 1..64 — vertex 0 (the config's query) + 64 sampled sources."""
+    """configs[0]: RMAT scale-16 ef16, w 1..64 — vertex 0 (isolated in the permuted ids), the
+    generator's vertex 0 (the config's query, reading N10) + 64 sampled sources."""
     c = gen.CONFIGS["c1"]
     src, dst, w = c.edges()
-    sources = np.concatenate([[0], gen.sample_sources(c.n, src, dst, 64, seed=42)]).astype(np.uint32)
+    sources = np.concatenate([[0, gen.generator_vertex(c, 0)], gen.sample_sources(c.n, src, dst, 64, seed=42)])
+    sources = sources.astype(np.uint32)
     _check_queries(c.n, src, dst, w, sources, K=20)
 
 
