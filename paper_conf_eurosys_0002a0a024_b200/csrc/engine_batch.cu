@@ -77,6 +77,15 @@ struct BParams {
     uint32_t K, KP;             // hubs in HB; row stride 2*KP (KP = K rounded up to a multiple of 4)
     int reduced;                // phase 2 starts with the certificate-driven pull (NEXT-1)
     uint32_t fresh;             // bit p-1: phase p pre-reads values from L2 instead of L1
+    // phase-1 pull over CG^R in SELL-32 (graph.hpp PullSell): dense iterations, no atomics
+    const uint32_t* pl_vtx;
+    const uint32_t* pl_deg;
+    const uint32_t* pl_soff;
+    const uint2* pl_tile;
+    const uint32_t* pl_adj;
+    const uint2* pl_adjw;
+    uint32_t pl_ntiles;
+    uint32_t pl_thr;            // pull a phase-1 iteration whose push would scan >= pl_thr edges (0: never)
     unsigned long long* trace;  // nullable: per iteration {t_start, t_s1, t_s2, phase<<62|q0<<32|listed, active<<32|edges}
     uint32_t trace_cap;
     unsigned long long* trace_cta;  // nullable: per iteration {first, last} CTA S2 finish times
@@ -112,6 +121,17 @@ struct Lanes32 {  // one u32 per query (Table 6 types), QN queries per pass, CGB
         if constexpr (VIT) return vit_arg(w);
         else return w;
     }
+    // owner-computes pull (phase 1, SELL CG^R): fold candidates into a register row, then merge
+    __device__ static uint32_t pid() { return O::INIT; }  // identity of the kind's select
+    __device__ static void fold(uint32_t& b, uint32_t u, const Arg& w) {
+        if (u == O::INIT) return;  // an unreached u has no candidate (SSSP / BFS would wrap)
+        uint32_t x;
+        if constexpr (VIT) x = vit_div(u, w);
+        else x = O::ext(u, w);
+        if (O::better(x, b)) b = x;
+    }
+    __device__ static uint32_t improve(uint32_t b, uint32_t c) { return O::better(b, c) ? 1u : 0u; }
+    __device__ static uint32_t merged(uint32_t b, uint32_t c) { return O::better(b, c) ? b : c; }
     // Process + EdgeFunction of G queries: candidates and Needed tests for all G without
     // branches, then one EdgeFunction per needed query (act: 4 query bits; an unreached u —
     // a pull may read one — is never Needed).
@@ -192,6 +212,21 @@ struct Lanes16 {
         const __half2 a = *reinterpret_cast<const __half2*>(&x), b = *reinterpret_cast<const __half2*>(&c);
         return MAXK ? __hgt2_mask(a, b) : __hlt2_mask(a, b);
     }
+    __device__ static uint32_t sel2(uint32_t x, uint32_t c) {  // the better of two words, per lane
+        const __half2 a = *reinterpret_cast<const __half2*>(&x), b = *reinterpret_cast<const __half2*>(&c);
+        const __half2 r = MAXK ? __hmax2(a, b) : __hmin2(a, b);
+        return *reinterpret_cast<const uint32_t*>(&r);
+    }
+    // owner-computes pull (phase 1, SELL CG^R): fold candidates into a register row, then merge
+    __device__ static uint32_t pid() { return init_word(); }
+    __device__ static void fold(uint32_t& b, uint32_t u, Arg w) {
+        b = sel2(b, ext2(u, (KIND == CG_BFS ? 0x3c00u : h16(w)) * 0x10001u));
+    }
+    __device__ static uint32_t improve(uint32_t b, uint32_t c) { return bits2(needed2(b, c)); }
+    __device__ static uint32_t merged(uint32_t b, uint32_t c) { return sel2(b, c); }
+    __device__ static bool overflow(uint32_t b, uint32_t c) {  // an improving lane reached 2048 (SSSP / BFS)
+        return (KIND == CG_SSSP || KIND == CG_BFS) && (__vcmpgeu2(b, LIMIT) & needed2(b, c)) != 0u;
+    }
     // Process + EdgeFunction of one 16 B chunk (4 words, 8 queries); act: 8 query bits.
     // The Needed test is taken on every lane, not only the active ones: a lane whose u is not
     // active for its query holds a value already pushed along (u, v), so its candidate is never
@@ -249,6 +284,10 @@ struct LanesBit {
     __device__ static void seed(uint32_t* p, uint32_t j, uint32_t) { atomicOr(p, 1u << j); }
     __device__ static uint32_t src_val() { return 1u; }
     __device__ static uint32_t nb_val(uint32_t) { return 1u; }
+    __device__ static uint32_t pid() { return 0u; }
+    __device__ static void fold(uint32_t& b, uint32_t u, uint32_t) { b |= u; }
+    __device__ static uint32_t improve(uint32_t b, uint32_t c) { return b & ~c; }
+    __device__ static uint32_t merged(uint32_t b, uint32_t c) { return b | c; }
     __device__ static uint32_t relax(uint32_t* p, const uint32_t (&u)[G], const uint32_t (&c)[G], uint32_t,
                                      uint32_t act, uint32_t& n_edges, uint32_t& n_upd, uint32_t*) {
         n_edges += __popc(act);
@@ -541,7 +580,7 @@ __device__ __forceinline__ void span_loads(const BParams& P, const GraphView& g,
 #define CGB_S1H 2
 #endif
 __device__ void compact_masks(const BParams& P, const GraphView& g, unsigned long long* cnt_slot,
-                              unsigned long long* act_slot, uint32_t* sm) {
+                              unsigned long long* act_slot, uint32_t* sm, uint32_t* wbuf, bool write_bits) {
     // One pass: the CTA's word range is taken in rounds of BW x H half-spans (H x 16 words =
     // H x 512 vertices per warp, all loads of a round issued together); a round's masks and
     // degrees stay in registers while the CTA reserves its list range (one 64-bit atomicAdd
@@ -615,9 +654,15 @@ __device__ void compact_masks(const BParams& P, const GraphView& g, unsigned lon
                     P.lo[i] = eb + incl - d;
                     P.lm[i] = mv[h][j];
                 }
+                if (lane == 0) wbuf[h * 16 + j] = bal;  // (the round's frontier words, below)
                 pos += __popc(bal);
                 eb += __shfl_sync(FULL, incl, 31);
             }
+        // phase-1 pull candidates: the bitmap = this frontier's vertices with edges, the "is u
+        // active" test of pull_sell (one coalesced store of the warp's 16 H words)
+        __syncwarp();
+        if (write_bits && lane < 16 * H && g0 + lane < w1) P.bitmap[g0 + lane] = wbuf[lane];
+        __syncwarp();
     }
     for (int o = 16; o > 0; o >>= 1) active += __shfl_xor_sync(FULL, active, o);
     if (lane == 0 && active) atomicAdd(act_slot, (unsigned long long)active);
@@ -1002,6 +1047,122 @@ __device__ void relax_pull(const BParams& P, uint32_t count, uint32_t E, uint32_
     }
 }
 
+// ------------------------------------------------------------------ phase-1 pull (owner computes)
+// One dense phase-1 iteration as a pull over CG^R in SELL-32 (graph.hpp PullSell): tile t of a
+// slice gives lane i the vertex v = vtx[32 s + i] and columns [c0, c0 + kPullTile) of its
+// in-edges (u -> v, w); for each u active in this iteration (bitmap bit, written by S1) the lane
+// folds the candidates of u's whole row (Table 6 (+) and select, every query lane: a lane not
+// active for u was already pushed along the edge, reading N6) into a register row; then it
+// compares with v's row and writes the improved words ONCE — a plain store by the owner (no
+// EdgeFunction atomics) unless the slice is split over several tiles (red.min / red.max).
+// v becomes active for the improved query lanes (M[v]).  Identical fixpoint: Alg 3's Process
+// applied in pull order (any order reaches the same unique values).
+template <int RW>
+__device__ __forceinline__ void row_load_ca(const uint32_t* p, uint32_t (&r)[RW]) {  // L1 may be stale: fine
+    if constexpr (RW % 4 == 0) {
+#pragma unroll
+        for (int i = 0; i < RW / 4; ++i) {
+            uint4 x;
+            asm volatile("ld.global.ca.v4.u32 {%0,%1,%2,%3}, [%4];"
+                         : "=r"(x.x), "=r"(x.y), "=r"(x.z), "=r"(x.w)
+                         : "l"(reinterpret_cast<const uint4*>(p) + i));
+            r[4 * i] = x.x, r[4 * i + 1] = x.y, r[4 * i + 2] = x.z, r[4 * i + 3] = x.w;
+        }
+    } else {
+#pragma unroll
+        for (int i = 0; i < RW; ++i) r[i] = ld_l1(p + i);
+    }
+}
+
+template <int KIND, bool PACKED, class L>
+__device__ void pull_sell(const BParams& P, uint32_t& n_edges, uint32_t& n_upd, uint32_t& n_read) {
+    constexpr int RW = L::RW;
+    constexpr uint32_t WM = L::QPW == 32 ? 0xffffffffu : (1u << L::QPW) - 1u;
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t gw = blockIdx.x * BW + (threadIdx.x >> 5);
+    const uint32_t NW = gridDim.x * BW;
+    const GraphView sg{nullptr, nullptr, P.pl_adj, P.pl_adjw};
+    auto active = [&](uint32_t u) { return (ld_l1(P.bitmap + (u >> 5)) >> (u & 31)) & 1u; };
+    for (uint32_t t = gw; t < P.pl_ntiles; t += NW) {
+        const uint2 tl = __ldg(P.pl_tile + t);  // (slice, first column)
+        const uint32_t v = __ldg(P.pl_vtx + tl.x * 32 + lane), d = __ldg(P.pl_deg + tl.x * 32 + lane);
+        const bool split = __shfl_sync(FULL, d, 0) > kPullTile;  // lane 0 holds the slice's widest row
+        const uint32_t c1 = min(tl.y + kPullTile, d);
+        const uint32_t base = __ldg(P.pl_soff + tl.x) + lane;
+        uint32_t best[RW];
+#pragma unroll
+        for (int i = 0; i < RW; ++i) best[i] = L::pid();
+        bool any = false;
+        uint32_t k = tl.y;
+        for (; k < c1; ++k) {
+            EdgeWord<PACKED> e0;
+            e0.load(sg, base + 32 * k);
+            uint32_t u0, w0;
+            e0.decode(P.dbits, P.dmask, u0, w0);
+            if (active(u0)) {
+                uint32_t r0[RW];
+                row_load_ca<RW>(P.V + (size_t)u0 * RW, r0);
+                const typename L::Arg a = L::arg(w0);
+#pragma unroll
+                for (int i = 0; i < RW; ++i) L::fold(best[i], r0[i], a);
+                any = true;
+                ++n_read;
+            }
+        }
+        if (!any) continue;
+        uint32_t* pv = P.V + (size_t)v * RW;
+        uint32_t cur[RW];
+        row_load_ca<RW>(pv, cur);  // (L1 holds no copy of v's row: only its owner touches it now)
+        uint32_t imp = 0, over = 0;
+#pragma unroll
+        for (int i = 0; i < RW; ++i) {
+            imp |= (L::improve(best[i], cur[i]) & WM) << (i * L::QPW);
+            if constexpr (L::QPW == 2) over |= (uint32_t)L::overflow(best[i], cur[i]);
+        }
+        if (over) atomicOr(P.err, ERR_LANE_OVERFLOW);
+        if (!imp) continue;
+        if (!split) {  // the owner's store of the merged row
+            if constexpr (RW % 4 == 0) {
+#pragma unroll
+                for (int i = 0; i < RW / 4; ++i)
+                    reinterpret_cast<uint4*>(pv)[i] = make_uint4(L::merged(best[4 * i], cur[4 * i]),
+                                                                 L::merged(best[4 * i + 1], cur[4 * i + 1]),
+                                                                 L::merged(best[4 * i + 2], cur[4 * i + 2]),
+                                                                 L::merged(best[4 * i + 3], cur[4 * i + 3]));
+            } else {
+#pragma unroll
+                for (int i = 0; i < RW; ++i) pv[i] = L::merged(best[i], cur[i]);
+            }
+            P.M[v] = imp;  // M[v] was consumed by S1: v is active for these queries
+        } else {  // a split slice: its tiles combine through the EdgeFunction
+            if constexpr (L::QPW == 2) {  // one 16 B vector EdgeFunction per 8 queries with an improved lane
+#pragma unroll
+                for (int h = 0; h < RW / 4; ++h) {
+                    if (!((imp >> (8 * h)) & 0xffu)) continue;
+                    if constexpr (KIND == CG_SSWP)
+                        asm volatile("red.relaxed.gpu.global.max.noftz.v4.f16x2 [%0], {%1,%2,%3,%4};" ::"l"(pv + 4 * h),
+                                     "r"(best[4 * h]), "r"(best[4 * h + 1]), "r"(best[4 * h + 2]), "r"(best[4 * h + 3])
+                                     : "memory");
+                    else
+                        asm volatile("red.relaxed.gpu.global.min.noftz.v4.f16x2 [%0], {%1,%2,%3,%4};" ::"l"(pv + 4 * h),
+                                     "r"(best[4 * h]), "r"(best[4 * h + 1]), "r"(best[4 * h + 2]), "r"(best[4 * h + 3])
+                                     : "memory");
+                }
+            } else {
+#pragma unroll
+                for (int i = 0; i < RW; ++i) {
+                    if (!((imp >> (i * L::QPW)) & WM)) continue;
+                    if constexpr (L::QPW == 32) red_or(pv + i, best[i]);
+                    else Op<KIND>::edge_fn(pv + i, best[i]);
+                }
+            }
+            red_or(P.M + v, imp);
+        }
+        n_upd += __popc(imp);
+        n_edges += __popc(imp);
+    }
+}
+
 // Batch-total count c (per thread) split evenly over the nq queries' counter k: block sum,
 // then thread 0 adds total/nq to each (the remainder to the first).
 __device__ __forceinline__ void block_add_split(unsigned long long* stats, int q0, int nq, int k, unsigned long long c,
@@ -1259,6 +1420,9 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
             }
             const unsigned long long t_s0 = (P.trace && tid == 0) ? global_ns() : 0ull;
             const int mode = pull ? F_UNCERT : predicate ? F_IMPACTED : bits ? F_BITS : F_MASKS;
+            // a dense phase-1 iteration may run as the owner-computes pull (pull_sell): its S1
+            // also leaves the frontier in the bitmap
+            const bool pcand = phase == 1 && P.pl_thr != 0u && mode == F_MASKS;
             if (mode == F_BITS) {
                 compact_bits(P, g, ctr + CT_LIST, ctr + CT_ACTIVE, sm_cnt);
             } else {
@@ -1266,7 +1430,7 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
                     mark_masks<KIND, L>(P, mode, sh, nq);
                     grid_sync(P.ctrl, epoch);
                 }
-                compact_masks(P, pull ? P.R : g, ctr + CT_LIST, ctr + CT_ACTIVE, sm_cnt);
+                compact_masks(P, pull ? P.R : g, ctr + CT_LIST, ctr + CT_ACTIVE, sm_cnt, xs, pcand);
             }
             grid_sync(P.ctrl, epoch);
             ++ring;
@@ -1326,10 +1490,14 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
                 relax_pull<KIND, PACKED, L>(P, count, E, xs, n_edges, n_upd, n_read);
                 pull = false;
                 bits = false;
+            } else if (pcand && E >= P.pl_thr) {  // dense phase-1 iteration: owner-computes pull
+                if constexpr (!InitOf<L>::ALL_ACTIVE) pull_sell<KIND, PACKED, L>(P, n_edges, n_upd, n_read);
+                bits = false;  // the next S1 reads the masks (and rewrites the bitmap)
             } else {
                 // small frontier: its S2 sets frontier bits (few reds) and the next S1 reads the
-                // bitmap; large frontier: no bitmap reds (they contend in L2), the next S1 scans M
-                bits = E < P.bits_below;  // at most E vertices change
+                // bitmap; large frontier: no bitmap reds (they contend in L2), the next S1 scans M.
+                // (A pull candidate's S1 left its frontier in the bitmap: no bitmap frontier next.)
+                bits = !pcand && E < P.bits_below;  // at most E vertices change
                 relax_b<KIND, PACKED, L>(P, g, count, E, xs, vs, bits, fresh, n_edges, n_upd, n_read,
                                          P.dyn ? ctr + CT_TILE : nullptr);
                 predicate = false;
@@ -1503,6 +1671,23 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
             P.HB = core.hub_vals.get();
             P.K = core.hub_k;
             P.KP = (core.hub_k + 3) & ~3u;
+        }
+    }
+    {   // phase-1 pull (pull_sell) over the kind's CG^R: iterations whose push would scan at least
+        // m_cg / CG_PULL_DIV edges (CG_PULL_DIV=0 disables it)
+        const char* e = getenv("CG_PULL_DIV");
+        const uint32_t div = e ? (uint32_t)strtoul(e, nullptr, 10) : 4u;
+        P.pl_thr = 0;
+        if (c.two_phase && c.cg && div && c.cg->pull.ntiles && c.kind != CG_WCC) {
+            const PullSell& S = c.cg->pull;
+            P.pl_vtx = S.vtx.get();
+            P.pl_deg = S.deg.get();
+            P.pl_soff = S.soff.get();
+            P.pl_tile = S.tile.get();
+            P.pl_adj = S.adj.get();
+            P.pl_adjw = S.adjw.get();
+            P.pl_ntiles = S.ntiles;
+            P.pl_thr = S.m_cg / div > 0 ? S.m_cg / div : 1u;
         }
     }
     P.srcs = c.srcs;
