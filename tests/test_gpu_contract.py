@@ -195,10 +195,10 @@ def test_calls_on_two_streams_are_ordered():
         g.build(k, K=16)
     ref = [to_np(g.query(k, to_dev(s))) for k, s in zip(kinds, srcs)]
     streams = [torch.cuda.Stream() for _ in range(2)]
+    sds = [to_dev(s) for s in srcs]  # kept alive until every stream is done (caching allocator)
+    torch.cuda.synchronize()
     outs = []
-    for i, (k, s) in enumerate(zip(kinds, srcs)):
-        sd = to_dev(s)
-        torch.cuda.current_stream().synchronize()
+    for i, (k, sd) in enumerate(zip(kinds, sds)):
         with torch.cuda.stream(streams[i % 2]):
             outs.append(g.query(k, sd))
     torch.cuda.synchronize()
