@@ -580,7 +580,10 @@ __device__ __forceinline__ void span_loads(const BParams& P, const GraphView& g,
 #define CGB_S1H 2
 #endif
 __device__ void compact_masks(const BParams& P, const GraphView& g, unsigned long long* cnt_slot,
-                              unsigned long long* act_slot, uint32_t* sm, uint32_t* wbuf, bool write_bits) {
+                              unsigned long long* act_slot, uint32_t* sm, uint32_t* wbuf, int bmode) {
+    // bmode 1: leave this frontier (vertices with edges) in the bitmap; 2: clear the bitmap words
+    const bool write_bits = bmode != 0;
+    const uint32_t wmask = bmode == 1 ? 0xffffffffu : 0u;
     // One pass: the CTA's word range is taken in rounds of BW x H half-spans (H x 16 words =
     // H x 512 vertices per warp, all loads of a round issued together); a round's masks and
     // degrees stay in registers while the CTA reserves its list range (one 64-bit atomicAdd
@@ -661,7 +664,7 @@ __device__ void compact_masks(const BParams& P, const GraphView& g, unsigned lon
         // phase-1 pull candidates: the bitmap = this frontier's vertices with edges, the "is u
         // active" test of pull_sell (one coalesced store of the warp's 16 H words)
         __syncwarp();
-        if (write_bits && lane < 16 * H && g0 + lane < w1) P.bitmap[g0 + lane] = wbuf[lane];
+        if (write_bits && lane < 16 * H && g0 + lane < w1) P.bitmap[g0 + lane] = wbuf[lane] & wmask;
         __syncwarp();
     }
     for (int o = 16; o > 0; o >>= 1) active += __shfl_xor_sync(FULL, active, o);
@@ -1403,6 +1406,8 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
         if (kt && q0 == 0) kt[1] = global_ns();
 
         int phase = P.two_phase ? 1 : 2;
+        uint32_t prevE = 0;      // the previous iteration's edges (pull candidacy)
+        bool bdirty = false;     // the bitmap holds a pull candidate's frontier (not a bitmap frontier)
         bool predicate = false;  // this iteration's S1 seeds Active with the impacted vertices
         bool bits = !InitOf<L>::ALL_ACTIVE;  // the frontier is in the bitmap (seeds set bits), else in M
         bool pull = false;       // this iteration is the NEXT-1 pull over uncertified vertices
@@ -1422,7 +1427,9 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
             const int mode = pull ? F_UNCERT : predicate ? F_IMPACTED : bits ? F_BITS : F_MASKS;
             // a dense phase-1 iteration may run as the owner-computes pull (pull_sell): its S1
             // also leaves the frontier in the bitmap
-            const bool pcand = phase == 1 && P.pl_thr != 0u && mode == F_MASKS;
+            const bool pcand = phase == 1 && P.pl_thr != 0u && mode == F_MASKS && prevE >= P.pl_thr / 2;
+            const int bmode = pcand ? 1 : (bdirty && mode != F_BITS) ? 2 : 0;
+            if (mode != F_BITS) bdirty = pcand;
             if (mode == F_BITS) {
                 compact_bits(P, g, ctr + CT_LIST, ctr + CT_ACTIVE, sm_cnt);
             } else {
@@ -1430,7 +1437,7 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
                     mark_masks<KIND, L>(P, mode, sh, nq);
                     grid_sync(P.ctrl, epoch);
                 }
-                compact_masks(P, pull ? P.R : g, ctr + CT_LIST, ctr + CT_ACTIVE, sm_cnt, xs, pcand);
+                compact_masks(P, pull ? P.R : g, ctr + CT_LIST, ctr + CT_ACTIVE, sm_cnt, xs, bmode);
             }
             grid_sync(P.ctrl, epoch);
             ++ring;
@@ -1491,17 +1498,18 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
                 pull = false;
                 bits = false;
             } else if (pcand && E >= P.pl_thr) {  // dense phase-1 iteration: owner-computes pull
-                if constexpr (!InitOf<L>::ALL_ACTIVE) pull_sell<KIND, PACKED, L>(P, n_edges, n_upd, n_read);
+                if constexpr (L::QPW == 32) pull_sell<KIND, PACKED, L>(P, n_edges, n_upd, n_read);
                 bits = false;  // the next S1 reads the masks (and rewrites the bitmap)
             } else {
                 // small frontier: its S2 sets frontier bits (few reds) and the next S1 reads the
                 // bitmap; large frontier: no bitmap reds (they contend in L2), the next S1 scans M.
                 // (A pull candidate's S1 left its frontier in the bitmap: no bitmap frontier next.)
-                bits = !pcand && E < P.bits_below;  // at most E vertices change
+                bits = !bdirty && E < P.bits_below;  // at most E vertices change
                 relax_b<KIND, PACKED, L>(P, g, count, E, xs, vs, bits, fresh, n_edges, n_upd, n_read,
                                          P.dyn ? ctr + CT_TILE : nullptr);
                 predicate = false;
             }
+            prevE = E;
             if (P.trace_cta && tr + 1 < P.trace_cap) {  // S2 load balance across CTAs (trace only)
                 __syncthreads();
                 if (threadIdx.x == 0) {
@@ -1675,10 +1683,12 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
     }
     {   // phase-1 pull (pull_sell) over the kind's CG^R: iterations whose push would scan at least
         // m_cg / CG_PULL_DIV edges (CG_PULL_DIV=0 disables it)
+        // default: REACH's bit lanes only (measured: the lane-per-vertex pull is latency-bound on
+        // 64 B value rows, faster than the push only for 4 B rows)
         const char* e = getenv("CG_PULL_DIV");
-        const uint32_t div = e ? (uint32_t)strtoul(e, nullptr, 10) : 4u;
+        const uint32_t div = e ? (uint32_t)strtoul(e, nullptr, 10) : 2u;
         P.pl_thr = 0;
-        if (c.two_phase && c.cg && div && c.cg->pull.ntiles && c.kind != CG_WCC) {
+        if (lw == 1 && c.two_phase && c.cg && div && c.cg->pull.ntiles && c.kind != CG_WCC) {
             const PullSell& S = c.cg->pull;
             P.pl_vtx = S.vtx.get();
             P.pl_deg = S.deg.get();
