@@ -14,7 +14,6 @@
 //      which is the edge the FIFO examines first; the next level is ordered by that key.
 //   a6 connectivity edges (Alg 1 l.8-12; reading Q8).
 //   a7 stream compaction of the flagged edges into the CG's CSR.
-#include <cub/device/device_radix_sort.cuh>
 #include <cub/device/device_scan.cuh>
 
 #include <chrono>
@@ -429,7 +428,7 @@ void alg2(Graph& G, const std::vector<uint32_t>& hubs, uint8_t* flags, bool per_
 
 namespace {
 
-// ---------------------------------------------------------------- CG^R in SELL-32 (phase-1 pull)
+// ---------------------------------------------------------------- CG^R (phase-1 pull)
 __global__ void k_cg_indeg(uint32_t n, GraphView cg, uint32_t dbits, uint32_t* __restrict__ indeg) {
     const uint32_t lane = threadIdx.x & 31;
     const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
@@ -441,99 +440,70 @@ __global__ void k_cg_indeg(uint32_t n, GraphView cg, uint32_t dbits, uint32_t* _
         }
 }
 
-__global__ void k_iota(uint32_t n, uint32_t* __restrict__ a) {
-    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
-        a[i] = (uint32_t)i;
-}
-
-// slot arrays of the sorted vertices (cnt of them have in-edges), their inverse map, widths
-__global__ void k_sell_slots(uint32_t n, uint32_t cnt, uint32_t nsl, const uint32_t* __restrict__ sdeg,
-                             const uint32_t* __restrict__ svtx, uint32_t* __restrict__ vtx, uint32_t* __restrict__ deg,
-                             uint32_t* __restrict__ slot, uint32_t* __restrict__ width) {
-    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < (uint64_t)nsl * 32;
-         i += (uint64_t)gridDim.x * blockDim.x) {
-        const bool ok = i < cnt;
-        vtx[i] = ok ? svtx[i] : 0xffffffffu;
-        deg[i] = ok ? sdeg[i] : 0u;
-        if (ok) slot[svtx[i]] = (uint32_t)i;
-        if (i % 32 == 0) width[i / 32] = sdeg[i];  // lane 0 holds the slice's largest in-degree
-    }
-}
-
-__global__ void k_sell_fill(uint32_t n, GraphView cg, uint32_t dbits, const uint32_t* __restrict__ slot,
-                            const uint32_t* __restrict__ soff, uint32_t* __restrict__ fill, uint32_t* __restrict__ sadj,
-                            uint2* __restrict__ sadjw) {
+// CG^R rows: in-edge (u -> v, w) stored in row v as u in G's edge encoding (order within a row is
+// immaterial: the pull's select is order-independent)
+__global__ void k_cg_rfill(uint32_t n, GraphView cg, uint32_t dbits, int packed, const uint32_t* __restrict__ rptr,
+                           uint32_t* __restrict__ fill, uint32_t* __restrict__ radj, uint2* __restrict__ radjw) {
     const uint32_t lane = threadIdx.x & 31;
     const uint64_t nw = (uint64_t)gridDim.x * (blockDim.x / 32);
     for (uint64_t u = blockIdx.x * (uint64_t)(blockDim.x / 32) + (threadIdx.x >> 5); u < n; u += nw)
         for (uint32_t e = cg.ptr[u] + lane; e < cg.end[u]; e += 32) {
             uint32_t v, w;
             edge_at(cg, e, dbits, v, w);
-            const uint32_t sl = slot[v];
-            const uint32_t k = atomicAdd(fill + v, 1u);
-            const size_t pos = (size_t)soff[sl / 32] + (size_t)k * 32 + (sl % 32);
-            if (sadj) sadj[pos] = (uint32_t)u | (dbits >= 32 ? 0u : (w - 1u) << dbits);
-            else sadjw[pos] = make_uint2((uint32_t)u, w);
+            const uint32_t pos = rptr[v] + atomicAdd(fill + v, 1u);
+            if (packed) radj[pos] = (uint32_t)u | ((w - 1u) << dbits);
+            else radjw[pos] = make_uint2((uint32_t)u, w);
         }
 }
 
+// the vertices with in-edges, in vertex order, and their first in-edge (flags -> positions)
+__global__ void k_pull_list(uint32_t n, const uint32_t* __restrict__ rptr, const uint32_t* __restrict__ pos,
+                            uint32_t* __restrict__ lv, uint32_t* __restrict__ lo) {
+    for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v < n; v += (uint64_t)gridDim.x * blockDim.x)
+        if (rptr[v + 1] > rptr[v]) {
+            lv[pos[v]] = (uint32_t)v;
+            lo[pos[v]] = rptr[v];
+        }
+}
+
+__global__ void k_has_in(uint32_t n, const uint32_t* __restrict__ indeg, uint32_t* __restrict__ flag) {
+    for (uint64_t v = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; v <= n; v += (uint64_t)gridDim.x * blockDim.x)
+        flag[v] = v < n && indeg[v] ? 1u : 0u;
+}
+
 void build_pull(Graph& G, Core& C, cudaStream_t s) {
-    PullSell& P = C.pull;
     const GraphView cg = core_view(G, C);
-    DevBuf<uint32_t> indeg(G.n ? G.n : 1, s), ids(G.n ? G.n : 1, s), sdeg(G.n ? G.n : 1, s),
-        svtx(G.n ? G.n : 1, s);
+    DevBuf<uint32_t> indeg(G.n + 1, s), pos(G.n + 1, s);
     CGB_CUDA(cudaMemsetAsync(indeg.get(), 0, indeg.bytes(), s));
     CGB_LAUNCH(k_cg_indeg, grid_rows(G.n), TB, 0, s, G.n, cg, G.dbits, indeg.get());
-    CGB_LAUNCH(k_iota, 4 * G.num_sms, TB, 0, s, G.n, ids.get());
-    size_t tmp = 0;
-    CGB_CUDA(cub::DeviceRadixSort::SortPairsDescending(nullptr, tmp, indeg.get(), sdeg.get(), ids.get(), svtx.get(),
-                                                       (int64_t)G.n, 0, 32, s));
-    {
-        DevBuf<uint8_t> t(tmp, s);
-        CGB_CUDA(cub::DeviceRadixSort::SortPairsDescending(t.get(), tmp, indeg.get(), sdeg.get(), ids.get(),
-                                                           svtx.get(), (int64_t)G.n, 0, 32, s));
-        count_launch(4);
-    }
-    // cnt = vertices with in-degree > 0 (a prefix of the sorted order), from the host copy
-    std::vector<uint32_t> h(G.n);
-    CGB_CUDA(cudaMemcpyAsync(h.data(), sdeg.get(), 4ull * G.n, cudaMemcpyDeviceToHost, s));
-    CGB_CUDA(cudaStreamSynchronize(s));
-    uint32_t cnt = 0;
-    while (cnt < G.n && h[cnt]) ++cnt;
-    P.nsl = (cnt + 31) / 32;
-    P.m_cg = C.m_cg;
-    std::vector<uint32_t> soff(P.nsl + 1, 0);
-    std::vector<uint2> tiles;
-    uint64_t tot = 0;
-    for (uint32_t sl = 0; sl < P.nsl; ++sl) {
-        const uint32_t wdt = h[(size_t)sl * 32];
-        soff[sl] = (uint32_t)tot;
-        tot += 32ull * wdt;
-        for (uint32_t c = 0; c < wdt; c += kPullTile) tiles.push_back(make_uint2(sl, c));
-    }
-    CGB_CHECK(tot < 0xffffffffull, CG_EOVERFLOW, "Core Graph too large for the pull layout");
-    P.ntiles = (uint32_t)tiles.size();
-    P.vtx.alloc((size_t)P.nsl * 32 + 1, s);
-    P.deg.alloc((size_t)P.nsl * 32 + 1, s);
-    P.soff.alloc(P.nsl + 1, s);
-    P.tile.alloc(P.ntiles + 1, s);
-    DevBuf<uint32_t> slot(G.n ? G.n : 1, s), width(P.nsl + 1, s);
-    if (P.nsl)
-        CGB_LAUNCH(k_sell_slots, 4 * G.num_sms, TB, 0, s, G.n, cnt, P.nsl, sdeg.get(), svtx.get(), P.vtx.get(),
-                   P.deg.get(), slot.get(), width.get());
-    CGB_CUDA(cudaMemcpyAsync(P.soff.get(), soff.data(), 4ull * (P.nsl + 1), cudaMemcpyHostToDevice, s));
-    if (P.ntiles) CGB_CUDA(cudaMemcpyAsync(P.tile.get(), tiles.data(), 8ull * P.ntiles, cudaMemcpyHostToDevice, s));
-    P.adj.reset();
-    P.adjw.reset();
-    if (G.packed) P.adj.alloc(adj_alloc_elems(tot, 4), s); else P.adjw.alloc(adj_alloc_elems(tot, 8), s);
+    C.rcg.n = G.n;
+    C.rcg.m = C.m_cg;
+    C.rcg.ptr.alloc(G.n + 1, s);
+    exclusive_sum(indeg.get(), C.rcg.ptr.get(), (uint64_t)G.n + 1, s);  // indeg[n] = 0
+    C.rcg.adj.reset();
+    C.rcg.adjw.reset();
+    if (G.packed) C.rcg.adj.alloc(adj_alloc_elems(C.m_cg, 4), s); else C.rcg.adjw.alloc(adj_alloc_elems(C.m_cg, 8), s);
+    CGB_LAUNCH(k_has_in, 4 * G.num_sms, TB, 0, s, G.n, indeg.get(), pos.get());
+    DevBuf<uint32_t> flag(G.n + 1, s);
+    CGB_CUDA(cudaMemcpyAsync(flag.get(), pos.get(), 4ull * (G.n + 1), cudaMemcpyDeviceToDevice, s));
+    exclusive_sum(flag.get(), pos.get(), (uint64_t)G.n + 1, s);
     CGB_CUDA(cudaMemsetAsync(indeg.get(), 0, indeg.bytes(), s));  // reused as the fill counters
-    CGB_LAUNCH(k_sell_fill, grid_rows(G.n), TB, 0, s, G.n, cg, G.packed ? G.dbits : 32u, slot.get(), P.soff.get(),
-               indeg.get(), P.adj.get(), P.adjw.get());
-    CGB_CUDA(cudaStreamSynchronize(s));  // h / soff / tiles (host) are released on return
+    CGB_LAUNCH(k_cg_rfill, grid_rows(G.n), TB, 0, s, G.n, cg, G.dbits, G.packed ? 1 : 0, C.rcg.ptr.get(), indeg.get(),
+               C.rcg.adj.get(), C.rcg.adjw.get());
+    uint32_t cnt = 0;
+    CGB_CUDA(cudaMemcpyAsync(&cnt, pos.get() + G.n, 4, cudaMemcpyDeviceToHost, s));
+    CGB_CUDA(cudaStreamSynchronize(s));
+    C.pl_count = cnt;
+    C.pl_v.alloc(cnt + 1, s);
+    C.pl_lo.alloc(cnt + 1, s);
+    CGB_LAUNCH(k_pull_list, 4 * G.num_sms, TB, 0, s, G.n, C.rcg.ptr.get(), pos.get(), C.pl_v.get(), C.pl_lo.get());
+    CGB_CUDA(cudaStreamSynchronize(s));
+    C.rcg_built = true;
 }
 
 // a7: the split rows from C.fbits
 void split_core(Graph& G, Core& C, cudaStream_t s) {
+    C.rcg_built = false;
     C.cg_end.alloc(G.n ? G.n : 1, s);
     C.sadj.reset();
     C.sadjw.reset();

@@ -77,14 +77,11 @@ struct BParams {
     uint32_t K, KP;             // hubs in HB; row stride 2*KP (KP = K rounded up to a multiple of 4)
     int reduced;                // phase 2 starts with the certificate-driven pull (NEXT-1)
     uint32_t fresh;             // bit p-1: phase p pre-reads values from L2 instead of L1
-    // phase-1 pull over CG^R in SELL-32 (graph.hpp PullSell): dense iterations, no atomics
-    const uint32_t* pl_vtx;
-    const uint32_t* pl_deg;
-    const uint32_t* pl_soff;
-    const uint2* pl_tile;
-    const uint32_t* pl_adj;
-    const uint2* pl_adjw;
-    uint32_t pl_ntiles;
+    // phase-1 pull over CG^R (relax_pull_all): dense iterations
+    GraphView RC;               // CG^R (in-edges of the Core Graph)
+    const uint32_t* pl_v;       // vertices with CG in-edges (vertex order) ...
+    const uint32_t* pl_lo;      // ... and their first in-edge in RC
+    uint32_t pl_count, pl_E;    // how many; |E_c|
     uint32_t pl_thr;            // pull a phase-1 iteration whose push would scan >= pl_thr edges (0: never)
     unsigned long long* trace;  // nullable: per iteration {t_start, t_s1, t_s2, phase<<62|q0<<32|listed, active<<32|edges}
     uint32_t trace_cap;
@@ -121,17 +118,14 @@ struct Lanes32 {  // one u32 per query (Table 6 types), QN queries per pass, CGB
         if constexpr (VIT) return vit_arg(w);
         else return w;
     }
-    // owner-computes pull (phase 1, SELL CG^R): fold candidates into a register row, then merge
-    __device__ static uint32_t pid() { return O::INIT; }  // identity of the kind's select
-    __device__ static void fold(uint32_t& b, uint32_t u, const Arg& w) {
-        if (u == O::INIT) return;  // an unreached u has no candidate (SSSP / BFS would wrap)
-        uint32_t x;
-        if constexpr (VIT) x = vit_div(u, w);
-        else x = O::ext(u, w);
-        if (O::better(x, b)) b = x;
+    // the pull (phase 1 over CG^R): one query's candidate from u's word, the select of two words
+    __device__ static uint32_t cand(uint32_t u, const Arg& w) {
+        if (u == O::INIT) return O::INIT;  // an unreached u has no candidate (SSSP / BFS would wrap)
+        if constexpr (VIT) return vit_div(u, w);
+        else return O::ext(u, w);
     }
+    __device__ static uint32_t sel(uint32_t a, uint32_t b) { return O::better(a, b) ? a : b; }
     __device__ static uint32_t improve(uint32_t b, uint32_t c) { return O::better(b, c) ? 1u : 0u; }
-    __device__ static uint32_t merged(uint32_t b, uint32_t c) { return O::better(b, c) ? b : c; }
     // Process + EdgeFunction of G queries: candidates and Needed tests for all G without
     // branches, then one EdgeFunction per needed query (act: 4 query bits; an unreached u —
     // a pull may read one — is never Needed).
@@ -217,13 +211,10 @@ struct Lanes16 {
         const __half2 r = MAXK ? __hmax2(a, b) : __hmin2(a, b);
         return *reinterpret_cast<const uint32_t*>(&r);
     }
-    // owner-computes pull (phase 1, SELL CG^R): fold candidates into a register row, then merge
-    __device__ static uint32_t pid() { return init_word(); }
-    __device__ static void fold(uint32_t& b, uint32_t u, Arg w) {
-        b = sel2(b, ext2(u, (KIND == CG_BFS ? 0x3c00u : h16(w)) * 0x10001u));
-    }
+    // the pull (phase 1 over CG^R): the candidates of u's word (+inf stays +inf), per-lane select
+    __device__ static uint32_t cand(uint32_t u, Arg w) { return ext2(u, (KIND == CG_BFS ? 0x3c00u : h16(w)) * 0x10001u); }
+    __device__ static uint32_t sel(uint32_t a, uint32_t b) { return sel2(a, b); }
     __device__ static uint32_t improve(uint32_t b, uint32_t c) { return bits2(needed2(b, c)); }
-    __device__ static uint32_t merged(uint32_t b, uint32_t c) { return sel2(b, c); }
     __device__ static bool overflow(uint32_t b, uint32_t c) {  // an improving lane reached 2048 (SSSP / BFS)
         return (KIND == CG_SSSP || KIND == CG_BFS) && (__vcmpgeu2(b, LIMIT) & needed2(b, c)) != 0u;
     }
@@ -284,10 +275,9 @@ struct LanesBit {
     __device__ static void seed(uint32_t* p, uint32_t j, uint32_t) { atomicOr(p, 1u << j); }
     __device__ static uint32_t src_val() { return 1u; }
     __device__ static uint32_t nb_val(uint32_t) { return 1u; }
-    __device__ static uint32_t pid() { return 0u; }
-    __device__ static void fold(uint32_t& b, uint32_t u, uint32_t) { b |= u; }
+    __device__ static uint32_t cand(uint32_t u, uint32_t) { return u; }
+    __device__ static uint32_t sel(uint32_t a, uint32_t b) { return a | b; }
     __device__ static uint32_t improve(uint32_t b, uint32_t c) { return b & ~c; }
-    __device__ static uint32_t merged(uint32_t b, uint32_t c) { return b | c; }
     __device__ static uint32_t relax(uint32_t* p, const uint32_t (&u)[G], const uint32_t (&c)[G], uint32_t,
                                      uint32_t act, uint32_t& n_edges, uint32_t& n_upd, uint32_t*) {
         n_edges += __popc(act);
@@ -580,10 +570,7 @@ __device__ __forceinline__ void span_loads(const BParams& P, const GraphView& g,
 #define CGB_S1H 2
 #endif
 __device__ void compact_masks(const BParams& P, const GraphView& g, unsigned long long* cnt_slot,
-                              unsigned long long* act_slot, uint32_t* sm, uint32_t* wbuf, int bmode) {
-    // bmode 1: leave this frontier (vertices with edges) in the bitmap; 2: clear the bitmap words
-    const bool write_bits = bmode != 0;
-    const uint32_t wmask = bmode == 1 ? 0xffffffffu : 0u;
+                              unsigned long long* act_slot, uint32_t* sm) {
     // One pass: the CTA's word range is taken in rounds of BW x H half-spans (H x 16 words =
     // H x 512 vertices per warp, all loads of a round issued together); a round's masks and
     // degrees stay in registers while the CTA reserves its list range (one 64-bit atomicAdd
@@ -657,15 +644,9 @@ __device__ void compact_masks(const BParams& P, const GraphView& g, unsigned lon
                     P.lo[i] = eb + incl - d;
                     P.lm[i] = mv[h][j];
                 }
-                if (lane == 0) wbuf[h * 16 + j] = bal;  // (the round's frontier words, below)
                 pos += __popc(bal);
                 eb += __shfl_sync(FULL, incl, 31);
             }
-        // phase-1 pull candidates: the bitmap = this frontier's vertices with edges, the "is u
-        // active" test of pull_sell (one coalesced store of the warp's 16 H words)
-        __syncwarp();
-        if (write_bits && lane < 16 * H && g0 + lane < w1) P.bitmap[g0 + lane] = wbuf[lane] & wmask;
-        __syncwarp();
     }
     for (int o = 16; o > 0; o >>= 1) active += __shfl_xor_sync(FULL, active, o);
     if (lane == 0 && active) atomicAdd(act_slot, (unsigned long long)active);
@@ -834,6 +815,220 @@ __device__ __forceinline__ void window_edges(const BParams& P, const GraphView& 
         }
     }
     cp_async_wait<0>();
+}
+
+// ------------------------------------------------------------------ phase-1 pull (dense iterations)
+// A dense phase-1 iteration as a pull over CG^R (Process, Alg 3 l.21-34, applied from the
+// destination's side): every in-edge (u -> v, w) of the Core Graph is relaxed; the window's 32 rows
+// are DESTINATIONS, held in xs as their current values, and a lane gathers the SOURCE row u (the
+// push pipeline's fetch / request, unchanged) and forms the candidates of all Q queries.  Lanes of
+// a chunk that share a destination are combined by a segmented warp scan (the kind's select, Table
+// 6); the last lane of each segment compares with the xs row and, where better, updates it and
+// applies the EdgeFunction ONCE for the row (vector red.min / red.max; red.or for REACH's bits) —
+// one atomic per (row, chunk) instead of one per (edge, query).  Every CG in-edge is read, active or
+// not: an inactive u's candidate was already applied to v (reading N6), so the extra candidates
+// change nothing.  v becomes active (M) for the improved queries.
+template <int KIND, bool PACKED, class L>
+__device__ __forceinline__ void window_pull(const BParams& P, const GraphView& g, uint32_t* xs, uint32_t* vs,
+                                            uint32_t off, uint32_t base, uint32_t vtx, uint32_t e, uint32_t ehi,
+                                            uint32_t& n_edges, uint32_t& n_upd, uint32_t& n_read) {
+    constexpr int EA = (L::QPW == 2 && E_AHEAD == S_PIPE) ? 2 * S_PIPE : E_AHEAD;
+    constexpr int S = S_PIPE, RW = L::RW;
+    constexpr uint32_t WM = L::QPW == 32 ? 0xffffffffu : (1u << L::QPW) - 1u;
+    using RC = RowCopy<L>;
+    constexpr uint32_t NONE = 0xffffffffu;
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t swz = RC::sw(lane);
+    if (e >= ehi) return;
+    const uint32_t nch = (ehi - e + 31) >> 5;
+    EdgeWord<PACKED> ew[EA];
+    uint32_t ek[EA];
+    uint32_t sw[S], sk[S];
+    auto fetch = [&](uint32_t c, EdgeWord<PACKED>& wd, uint32_t& kout) {
+        const uint32_t cs = e + c * 32, t = cs + lane;
+        const uint32_t below = __popc(__ballot_sync(FULL, off <= cs));
+        const uint32_t rel = off - cs;
+        const uint32_t starts = __reduce_or_sync(FULL, (rel - 1u < 31u) ? (1u << rel) : 0u);
+        const uint32_t kk = below - 1u + __popc(starts & ((2u << lane) - 1u));
+        const uint32_t a = __shfl_sync(FULL, base, kk) + t;
+        const bool ok = t < ehi;
+        if (ok) wd.load(g, a);
+        kout = ok ? kk : NONE;
+    };
+    auto request = [&](int slot, const EdgeWord<PACKED>& wd, uint32_t kk) {
+        sk[slot] = kk;
+        uint32_t dd = NONE;
+        if (kk != NONE) {
+            uint32_t d, w;
+            wd.decode(P.dbits, P.dmask, d, w);  // d = the source u of the in-edge
+            sw[slot] = w;
+            dd = d;
+        }
+        if constexpr (RC::C > 1) {
+            constexpr uint32_t RPI = 32 / RC::C;
+            const uint32_t p = lane % RC::C;
+#pragma unroll
+            for (uint32_t i = 0; i < RC::C; ++i) {
+                const uint32_t r = i * RPI + lane / RC::C;
+                const uint32_t dr = __shfl_sync(FULL, dd, r);
+                if (dr != NONE)
+                    RC::copy(vs + (slot * 32 + r) * RW + RC::CW4 * (p ^ RC::sw(r)), P.V + (size_t)dr * RW + RC::CW4 * p,
+                             false);
+            }
+        } else if (dd != NONE) {
+            RC::copy(vs + (slot * 32 + lane) * RW, P.V + (size_t)dd * RW, false);
+        }
+        cp_async_commit();
+    };
+#pragma unroll
+    for (int s = 0; s < EA; ++s) {
+        ek[s] = NONE;
+        if ((uint32_t)s < nch) fetch(s, ew[s], ek[s]);
+    }
+#pragma unroll
+    for (int s = 0; s < S - 1; ++s) {
+        request(s, ew[s], ek[s]);
+        ek[s] = NONE;
+        if ((uint32_t)(s + EA) < nch) fetch(s + EA, ew[s], ek[s]);
+    }
+    for (uint32_t c0 = 0; c0 < nch; c0 += EA) {
+#pragma unroll
+        for (int s = 0; s < EA; ++s) {
+            const uint32_t cc = c0 + s;
+            if (cc >= nch) break;
+            const int je = (s + S - 1) % EA;
+            const int jr = (s + S - 1) % S;
+            if constexpr (RC::C > 1) __syncwarp();
+            request(jr, ew[je], ek[je]);
+            ek[je] = NONE;
+            if (cc + S - 1 + EA < nch) fetch(cc + S - 1 + EA, ew[je], ek[je]);
+            cp_async_wait<S - 1>();
+            if constexpr (RC::C > 1) __syncwarp();
+            const int sr = s % S;
+            const uint32_t kk = sk[sr];
+            // the candidates of this lane's in-edge for every query
+            uint32_t x[RW];
+            {
+                const typename L::Arg w = L::arg(sw[sr]);
+                const uint32_t* rv = vs + (sr * 32 + lane) * RW;
+#pragma unroll
+                for (int i = 0; i < RW; ++i)
+                    x[i] = kk != NONE ? L::cand(rv[((i / RC::CW4) ^ swz) * RC::CW4 + i % RC::CW4], w) : 0u;
+            }
+            if (kk != NONE) ++n_read;
+            // segmented scan (the kind's select) over the lanes of each destination row
+#pragma unroll
+            for (uint32_t dl = 1; dl < 32; dl <<= 1) {
+                const uint32_t kd = __shfl_up_sync(FULL, kk, dl);
+                const bool take = lane >= dl && kd == kk;
+#pragma unroll
+                for (int i = 0; i < RW; ++i) {
+                    const uint32_t y = __shfl_up_sync(FULL, x[i], dl);
+                    if (take) x[i] = L::sel(x[i], y);
+                }
+            }
+            const uint32_t knext = __shfl_down_sync(FULL, kk, 1);
+            const uint32_t vk = __shfl_sync(FULL, vtx, kk & 31u);
+            const bool leader = kk != NONE && (lane == 31 || knext != kk);
+            if (leader) {
+                uint32_t* row = xs + kk * RW;
+                uint32_t* pv = P.V + (size_t)vk * RW;
+                uint32_t imp = 0, over = 0;
+#pragma unroll
+                for (int i = 0; i < RW; ++i) {
+                    const uint32_t c = row[i];
+                    const uint32_t im = L::improve(x[i], c) & WM;
+                    imp |= im << (i * L::QPW);
+                    if constexpr (L::QPW == 2) over |= (uint32_t)L::overflow(x[i], c);
+                    if (im) row[i] = L::sel(x[i], c);
+                }
+                if (over) atomicOr(P.err, ERR_LANE_OVERFLOW);
+                if (imp) {  // the row's EdgeFunction, once
+                    if constexpr (L::QPW == 2) {
+#pragma unroll
+                        for (int h = 0; h < RW / 4; ++h) {
+                            if (!((imp >> (8 * h)) & 0xffu)) continue;
+                            if constexpr (KIND == CG_SSWP)
+                                asm volatile("red.relaxed.gpu.global.max.noftz.v4.f16x2 [%0], {%1,%2,%3,%4};" ::"l"(pv + 4 * h),
+                                             "r"(x[4 * h]), "r"(x[4 * h + 1]), "r"(x[4 * h + 2]), "r"(x[4 * h + 3]) : "memory");
+                            else
+                                asm volatile("red.relaxed.gpu.global.min.noftz.v4.f16x2 [%0], {%1,%2,%3,%4};" ::"l"(pv + 4 * h),
+                                             "r"(x[4 * h]), "r"(x[4 * h + 1]), "r"(x[4 * h + 2]), "r"(x[4 * h + 3]) : "memory");
+                        }
+                    } else {
+#pragma unroll
+                        for (int i = 0; i < RW; ++i) {
+                            if (!((imp >> (i * L::QPW)) & WM)) continue;
+                            if constexpr (L::QPW == 32) red_or(pv + i, x[i]);
+                            else Op<KIND>::edge_fn(pv + i, x[i]);
+                        }
+                    }
+                    red_or(P.M + vk, imp);
+                    n_upd += __popc(imp);
+                    n_edges += __popc(imp);
+                }
+            }
+            __syncwarp();  // the leaders' xs updates are seen by the next chunk
+        }
+    }
+    cp_async_wait<0>();
+}
+
+// The whole in-edge list of CG^R (static: vertices with CG in-edges, vertex order) split evenly over
+// all warps; windows of 32 destinations as in relax_range.
+template <int KIND, bool PACKED, class L>
+__device__ void relax_pull_all(const BParams& P, uint32_t* xs, uint32_t* vs, uint32_t& n_edges, uint32_t& n_upd,
+                               uint32_t& n_read) {
+    constexpr int RW = L::RW;
+    using RC = RowCopy<L>;
+    const GraphView& g = P.RC;
+    const uint32_t count = P.pl_count, E = P.pl_E;
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t gw = blockIdx.x * BW + (threadIdx.x >> 5);
+    const uint64_t NW = (uint64_t)gridDim.x * BW;
+    const uint32_t e0 = (uint32_t)((uint64_t)E * gw / NW), e1 = (uint32_t)((uint64_t)E * (gw + 1) / NW);
+    if (e0 >= e1) return;
+    uint32_t lo = 0, hi = count;  // 32-ary search: the window holding edge e0
+    while (hi - lo > 32) {
+        const uint32_t step = (hi - lo + 31) / 32;
+        const uint32_t p = lo + lane * step;
+        const bool le = p < hi && __ldg(P.pl_lo + p) <= e0;
+        const uint32_t k = 31 - __clz(__ballot_sync(FULL, le));
+        const uint32_t nlo = lo + k * step;
+        hi = min(hi, nlo + step);
+        lo = nlo;
+    }
+    {
+        const uint32_t p = lo + lane;
+        const bool le = p < hi && __ldg(P.pl_lo + p) <= e0;
+        lo += 31 - __clz(__ballot_sync(FULL, le));
+    }
+    uint32_t i = lo, e = e0;
+    for (;;) {
+        const uint32_t idx = i + lane;
+        uint32_t v = 0, off = E;
+        if (idx < count) {
+            v = __ldg(P.pl_v + idx);
+            off = __ldg(P.pl_lo + idx);
+        }
+        __syncwarp();
+#pragma unroll
+        for (uint32_t r = 0; r < RC::C; ++r) {  // the window's destination rows -> xs
+            const uint32_t f = r * 32 + lane, row = f / RC::C, c = f % RC::C;
+            const uint32_t vr = __shfl_sync(FULL, v, row);
+            if (i + row < count) RC::copy(xs + row * RW + c * RC::CW4, P.V + (size_t)vr * RW + c * RC::CW4, true);
+        }
+        cp_async_commit();
+        cp_async_wait<0>();
+        __syncwarp();
+        const uint32_t wend = (i + 32 < count) ? __ldg(P.pl_lo + i + 32) : E;
+        const uint32_t ehi = min(e1, wend);
+        window_pull<KIND, PACKED, L>(P, g, xs, vs, off, 0u, v, e, ehi, n_edges, n_upd, n_read);
+        __syncwarp();
+        if (ehi >= e1) break;
+        e = ehi;
+        i += 32;
+    }
 }
 
 // The window's 32 rows (all Q queries) into shared memory, coalesced (RW words per row)
@@ -1047,122 +1242,6 @@ __device__ void relax_pull(const BParams& P, uint32_t count, uint32_t E, uint32_
         if (ehi >= e1) break;
         e = ehi;
         i += 32;
-    }
-}
-
-// ------------------------------------------------------------------ phase-1 pull (owner computes)
-// One dense phase-1 iteration as a pull over CG^R in SELL-32 (graph.hpp PullSell): tile t of a
-// slice gives lane i the vertex v = vtx[32 s + i] and columns [c0, c0 + kPullTile) of its
-// in-edges (u -> v, w); for each u active in this iteration (bitmap bit, written by S1) the lane
-// folds the candidates of u's whole row (Table 6 (+) and select, every query lane: a lane not
-// active for u was already pushed along the edge, reading N6) into a register row; then it
-// compares with v's row and writes the improved words ONCE — a plain store by the owner (no
-// EdgeFunction atomics) unless the slice is split over several tiles (red.min / red.max).
-// v becomes active for the improved query lanes (M[v]).  Identical fixpoint: Alg 3's Process
-// applied in pull order (any order reaches the same unique values).
-template <int RW>
-__device__ __forceinline__ void row_load_ca(const uint32_t* p, uint32_t (&r)[RW]) {  // L1 may be stale: fine
-    if constexpr (RW % 4 == 0) {
-#pragma unroll
-        for (int i = 0; i < RW / 4; ++i) {
-            uint4 x;
-            asm volatile("ld.global.ca.v4.u32 {%0,%1,%2,%3}, [%4];"
-                         : "=r"(x.x), "=r"(x.y), "=r"(x.z), "=r"(x.w)
-                         : "l"(reinterpret_cast<const uint4*>(p) + i));
-            r[4 * i] = x.x, r[4 * i + 1] = x.y, r[4 * i + 2] = x.z, r[4 * i + 3] = x.w;
-        }
-    } else {
-#pragma unroll
-        for (int i = 0; i < RW; ++i) r[i] = ld_l1(p + i);
-    }
-}
-
-template <int KIND, bool PACKED, class L>
-__device__ void pull_sell(const BParams& P, uint32_t& n_edges, uint32_t& n_upd, uint32_t& n_read) {
-    constexpr int RW = L::RW;
-    constexpr uint32_t WM = L::QPW == 32 ? 0xffffffffu : (1u << L::QPW) - 1u;
-    const uint32_t lane = threadIdx.x & 31;
-    const uint32_t gw = blockIdx.x * BW + (threadIdx.x >> 5);
-    const uint32_t NW = gridDim.x * BW;
-    const GraphView sg{nullptr, nullptr, P.pl_adj, P.pl_adjw};
-    auto active = [&](uint32_t u) { return (ld_l1(P.bitmap + (u >> 5)) >> (u & 31)) & 1u; };
-    for (uint32_t t = gw; t < P.pl_ntiles; t += NW) {
-        const uint2 tl = __ldg(P.pl_tile + t);  // (slice, first column)
-        const uint32_t v = __ldg(P.pl_vtx + tl.x * 32 + lane), d = __ldg(P.pl_deg + tl.x * 32 + lane);
-        const bool split = __shfl_sync(FULL, d, 0) > kPullTile;  // lane 0 holds the slice's widest row
-        const uint32_t c1 = min(tl.y + kPullTile, d);
-        const uint32_t base = __ldg(P.pl_soff + tl.x) + lane;
-        uint32_t best[RW];
-#pragma unroll
-        for (int i = 0; i < RW; ++i) best[i] = L::pid();
-        bool any = false;
-        uint32_t k = tl.y;
-        for (; k < c1; ++k) {
-            EdgeWord<PACKED> e0;
-            e0.load(sg, base + 32 * k);
-            uint32_t u0, w0;
-            e0.decode(P.dbits, P.dmask, u0, w0);
-            if (active(u0)) {
-                uint32_t r0[RW];
-                row_load_ca<RW>(P.V + (size_t)u0 * RW, r0);
-                const typename L::Arg a = L::arg(w0);
-#pragma unroll
-                for (int i = 0; i < RW; ++i) L::fold(best[i], r0[i], a);
-                any = true;
-                ++n_read;
-            }
-        }
-        if (!any) continue;
-        uint32_t* pv = P.V + (size_t)v * RW;
-        uint32_t cur[RW];
-        row_load_ca<RW>(pv, cur);  // (L1 holds no copy of v's row: only its owner touches it now)
-        uint32_t imp = 0, over = 0;
-#pragma unroll
-        for (int i = 0; i < RW; ++i) {
-            imp |= (L::improve(best[i], cur[i]) & WM) << (i * L::QPW);
-            if constexpr (L::QPW == 2) over |= (uint32_t)L::overflow(best[i], cur[i]);
-        }
-        if (over) atomicOr(P.err, ERR_LANE_OVERFLOW);
-        if (!imp) continue;
-        if (!split) {  // the owner's store of the merged row
-            if constexpr (RW % 4 == 0) {
-#pragma unroll
-                for (int i = 0; i < RW / 4; ++i)
-                    reinterpret_cast<uint4*>(pv)[i] = make_uint4(L::merged(best[4 * i], cur[4 * i]),
-                                                                 L::merged(best[4 * i + 1], cur[4 * i + 1]),
-                                                                 L::merged(best[4 * i + 2], cur[4 * i + 2]),
-                                                                 L::merged(best[4 * i + 3], cur[4 * i + 3]));
-            } else {
-#pragma unroll
-                for (int i = 0; i < RW; ++i) pv[i] = L::merged(best[i], cur[i]);
-            }
-            P.M[v] = imp;  // M[v] was consumed by S1: v is active for these queries
-        } else {  // a split slice: its tiles combine through the EdgeFunction
-            if constexpr (L::QPW == 2) {  // one 16 B vector EdgeFunction per 8 queries with an improved lane
-#pragma unroll
-                for (int h = 0; h < RW / 4; ++h) {
-                    if (!((imp >> (8 * h)) & 0xffu)) continue;
-                    if constexpr (KIND == CG_SSWP)
-                        asm volatile("red.relaxed.gpu.global.max.noftz.v4.f16x2 [%0], {%1,%2,%3,%4};" ::"l"(pv + 4 * h),
-                                     "r"(best[4 * h]), "r"(best[4 * h + 1]), "r"(best[4 * h + 2]), "r"(best[4 * h + 3])
-                                     : "memory");
-                    else
-                        asm volatile("red.relaxed.gpu.global.min.noftz.v4.f16x2 [%0], {%1,%2,%3,%4};" ::"l"(pv + 4 * h),
-                                     "r"(best[4 * h]), "r"(best[4 * h + 1]), "r"(best[4 * h + 2]), "r"(best[4 * h + 3])
-                                     : "memory");
-                }
-            } else {
-#pragma unroll
-                for (int i = 0; i < RW; ++i) {
-                    if (!((imp >> (i * L::QPW)) & WM)) continue;
-                    if constexpr (L::QPW == 32) red_or(pv + i, best[i]);
-                    else Op<KIND>::edge_fn(pv + i, best[i]);
-                }
-            }
-            red_or(P.M + v, imp);
-        }
-        n_upd += __popc(imp);
-        n_edges += __popc(imp);
     }
 }
 
@@ -1406,8 +1485,6 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
         if (kt && q0 == 0) kt[1] = global_ns();
 
         int phase = P.two_phase ? 1 : 2;
-        uint32_t prevE = 0;      // the previous iteration's edges (pull candidacy)
-        bool bdirty = false;     // the bitmap holds a pull candidate's frontier (not a bitmap frontier)
         bool predicate = false;  // this iteration's S1 seeds Active with the impacted vertices
         bool bits = !InitOf<L>::ALL_ACTIVE;  // the frontier is in the bitmap (seeds set bits), else in M
         bool pull = false;       // this iteration is the NEXT-1 pull over uncertified vertices
@@ -1425,11 +1502,6 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
             }
             const unsigned long long t_s0 = (P.trace && tid == 0) ? global_ns() : 0ull;
             const int mode = pull ? F_UNCERT : predicate ? F_IMPACTED : bits ? F_BITS : F_MASKS;
-            // a dense phase-1 iteration may run as the owner-computes pull (pull_sell): its S1
-            // also leaves the frontier in the bitmap
-            const bool pcand = phase == 1 && P.pl_thr != 0u && mode == F_MASKS && prevE >= P.pl_thr / 2;
-            const int bmode = pcand ? 1 : (bdirty && mode != F_BITS) ? 2 : 0;
-            if (mode != F_BITS) bdirty = pcand;
             if (mode == F_BITS) {
                 compact_bits(P, g, ctr + CT_LIST, ctr + CT_ACTIVE, sm_cnt);
             } else {
@@ -1437,7 +1509,7 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
                     mark_masks<KIND, L>(P, mode, sh, nq);
                     grid_sync(P.ctrl, epoch);
                 }
-                compact_masks(P, pull ? P.R : g, ctr + CT_LIST, ctr + CT_ACTIVE, sm_cnt, xs, bmode);
+                compact_masks(P, pull ? P.R : g, ctr + CT_LIST, ctr + CT_ACTIVE, sm_cnt);
             }
             grid_sync(P.ctrl, epoch);
             ++ring;
@@ -1497,19 +1569,17 @@ __global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
                 relax_pull<KIND, PACKED, L>(P, count, E, xs, n_edges, n_upd, n_read);
                 pull = false;
                 bits = false;
-            } else if (pcand && E >= P.pl_thr) {  // dense phase-1 iteration: owner-computes pull
-                if constexpr (L::QPW == 32) pull_sell<KIND, PACKED, L>(P, n_edges, n_upd, n_read);
-                bits = false;  // the next S1 reads the masks (and rewrites the bitmap)
+            } else if (phase == 1 && P.pl_thr != 0u && E >= P.pl_thr) {  // dense phase-1 iteration: pull
+                if constexpr (!InitOf<L>::ALL_ACTIVE) relax_pull_all<KIND, PACKED, L>(P, xs, vs, n_edges, n_upd, n_read);
+                bits = false;  // the pull marks the next frontier in M
             } else {
                 // small frontier: its S2 sets frontier bits (few reds) and the next S1 reads the
-                // bitmap; large frontier: no bitmap reds (they contend in L2), the next S1 scans M.
-                // (A pull candidate's S1 left its frontier in the bitmap: no bitmap frontier next.)
-                bits = !bdirty && E < P.bits_below;  // at most E vertices change
+                // bitmap; large frontier: no bitmap reds (they contend in L2), the next S1 scans M
+                bits = E < P.bits_below;  // at most E vertices change
                 relax_b<KIND, PACKED, L>(P, g, count, E, xs, vs, bits, fresh, n_edges, n_upd, n_read,
                                          P.dyn ? ctr + CT_TILE : nullptr);
                 predicate = false;
             }
-            prevE = E;
             if (P.trace_cta && tr + 1 < P.trace_cap) {  // S2 load balance across CTAs (trace only)
                 __syncthreads();
                 if (threadIdx.x == 0) {
@@ -1681,23 +1751,19 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
             P.KP = (core.hub_k + 3) & ~3u;
         }
     }
-    {   // phase-1 pull (pull_sell) over the kind's CG^R: iterations whose push would scan at least
-        // m_cg / CG_PULL_DIV edges (CG_PULL_DIV=0 disables it)
-        // default: REACH's bit lanes only (measured: the lane-per-vertex pull is latency-bound on
-        // 64 B value rows, faster than the push only for 4 B rows)
+    {   // phase-1 pull (relax_pull_all) over the kind's CG^R: iterations whose push would scan at
+        // least m_cg / CG_PULL_DIV edges (CG_PULL_DIV=0 disables it)
         const char* e = getenv("CG_PULL_DIV");
         const uint32_t div = e ? (uint32_t)strtoul(e, nullptr, 10) : 2u;
         P.pl_thr = 0;
-        if (lw == 1 && c.two_phase && c.cg && div && c.cg->pull.ntiles && c.kind != CG_WCC) {
-            const PullSell& S = c.cg->pull;
-            P.pl_vtx = S.vtx.get();
-            P.pl_deg = S.deg.get();
-            P.pl_soff = S.soff.get();
-            P.pl_tile = S.tile.get();
-            P.pl_adj = S.adj.get();
-            P.pl_adjw = S.adjw.get();
-            P.pl_ntiles = S.ntiles;
-            P.pl_thr = S.m_cg / div > 0 ? S.m_cg / div : 1u;
+        if (c.two_phase && c.cg && div && c.cg->rcg_built && c.kind != CG_WCC) {
+            const Core& C = *c.cg;
+            P.RC = view(C.rcg);
+            P.pl_v = C.pl_v.get();
+            P.pl_lo = C.pl_lo.get();
+            P.pl_count = C.pl_count;
+            P.pl_E = C.rcg.m;
+            P.pl_thr = C.rcg.m / div > 0 ? C.rcg.m / div : 1u;
         }
     }
     P.srcs = c.srcs;

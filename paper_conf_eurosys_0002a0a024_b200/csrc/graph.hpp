@@ -45,23 +45,6 @@ inline GraphView view(const Adj& a) { return GraphView{a.ptr.get(), nullptr, a.a
 // Phase 1 reads the CG rows, phase 2's first sweep the non-CG rows [cg_end[v], ptr[v+1])
 // (reading N7), later phase-2 iterations whole rows.  E_c membership in G's canonical edge
 // order is kept as a bitmap (cg_core_export, persistence, WCC).
-// CG^R in SELL-32-sigma form (sliced ELLPACK: vertices with CG in-edges sorted by in-degree,
-// descending, in slices of 32; slice s stores its in-edges column-major, edge k of lane i at
-// soff[s] + 32 k + i), for the owner-computes pull of dense phase-1 iterations: each lane folds
-// its vertex's in-edges into a value row in registers and writes the row once — no atomics.
-// A slice wider than kPullTile columns is split into several tiles whose partial rows are
-// combined with red.min / red.max.  Edge words are the source u, in G's packed / wide encoding.
-constexpr uint32_t kPullTile = 32;  // columns per tile
-struct PullSell {
-    uint32_t nsl = 0, ntiles = 0, m_cg = 0;
-    DevBuf<uint32_t> vtx;    // [nsl*32] vertex of (slice, lane); 0xFFFFFFFF past the last vertex
-    DevBuf<uint32_t> deg;    // [nsl*32] its CG in-degree (0 for padding lanes)
-    DevBuf<uint32_t> soff;   // [nsl] edge offset of slice s's column 0
-    DevBuf<uint2> tile;      // [ntiles] (slice, first column) of each tile of <= kPullTile columns
-    DevBuf<uint32_t> adj;    // SELL edge words (packed) ...
-    DevBuf<uint2> adjw;      // ... or (u, w) pairs (wide layout)
-};
-
 struct Core {
     bool built = false;
     int alg = 0;           // 1 = Algorithm 1 (specialized), 2 = Algorithm 2 (general)
@@ -79,7 +62,13 @@ struct Core {
     uint32_t hub_k = 0;
     Adj sym;               // WCC: CG ∪ CG^R (built on the first WCC 2Phase query)
     bool sym_built = false;
-    PullSell pull;         // CG^R for the phase-1 pull (built with the CG)
+    // CG^R for the pull of dense phase-1 iterations (engine_batch.cu relax_pull_all): the CSR of
+    // the reversed Core Graph, and the vertices with CG in-edges (vertex order) with their first
+    // in-edge — a static edge-offset list for the edge-balanced split
+    Adj rcg;
+    DevBuf<uint32_t> pl_v, pl_lo;
+    uint32_t pl_count = 0;
+    bool rcg_built = false;
 };
 
 struct Workspace {
