@@ -817,6 +817,9 @@ __device__ __forceinline__ void window_edges(const BParams& P, const GraphView& 
     cp_async_wait<0>();
 }
 
+template <class L>  // 128 B rows (RW = 32): one window buffer, so 16 warps' buffers fit in shared memory
+constexpr bool xs_double() { return L::RW <= 16; }
+
 // ------------------------------------------------------------------ phase-1 pull (dense iterations)
 // A dense phase-1 iteration as a pull over CG^R (Process, Alg 3 l.21-34, applied from the
 // destination's side): every in-edge (u -> v, w) of the Core Graph is relaxed; the window's 32 rows
@@ -1003,31 +1006,53 @@ __device__ void relax_pull_all(const BParams& P, uint32_t* xs, uint32_t* vs, uin
         const bool le = p < hi && __ldg(P.pl_lo + p) <= e0;
         lo += 31 - __clz(__ballot_sync(FULL, le));
     }
-    uint32_t i = lo, e = e0;
-    for (;;) {
-        const uint32_t idx = i + lane;
-        uint32_t v = 0, off = E;
+    auto list_load = [&](uint32_t i0, uint32_t& v, uint32_t& off) {
+        const uint32_t idx = i0 + lane;
+        v = 0;
+        off = E;
         if (idx < count) {
             v = __ldg(P.pl_v + idx);
             off = __ldg(P.pl_lo + idx);
         }
-        __syncwarp();
+    };
+    auto rows_async = [&](uint32_t* buf, uint32_t v, uint32_t i0) {  // the window's destination rows -> buf
 #pragma unroll
-        for (uint32_t r = 0; r < RC::C; ++r) {  // the window's destination rows -> xs
+        for (uint32_t r = 0; r < RC::C; ++r) {
             const uint32_t f = r * 32 + lane, row = f / RC::C, c = f % RC::C;
             const uint32_t vr = __shfl_sync(FULL, v, row);
-            if (i + row < count) RC::copy(xs + row * RW + c * RC::CW4, P.V + (size_t)vr * RW + c * RC::CW4, true);
+            if (i0 + row < count) RC::copy(buf + row * RW + c * RC::CW4, P.V + (size_t)vr * RW + c * RC::CW4, true);
         }
         cp_async_commit();
-        cp_async_wait<0>();
-        __syncwarp();
-        const uint32_t wend = (i + 32 < count) ? __ldg(P.pl_lo + i + 32) : E;
+    };
+    constexpr bool DB = xs_double<L>();  // the next window's rows are copied while this one runs
+    uint32_t i = lo, e = e0, cv, coff, nv, noff;
+    list_load(i, cv, coff);
+    rows_async(xs, cv, i);
+    list_load(i + 32, nv, noff);
+    uint32_t buf = 0;
+    for (;;) {
+        const uint32_t wend = (i + 32 < count) ? __shfl_sync(FULL, noff, 0) : E;
         const uint32_t ehi = min(e1, wend);
-        window_pull<KIND, PACKED, L>(P, g, xs, vs, off, 0u, v, e, ehi, n_edges, n_upd, n_read);
+        const bool more = ehi < e1;
+        uint32_t mv = 0, moff = E;
+        if (more) {
+            if constexpr (DB) rows_async(xs + (buf ^ 1) * 32 * RW, nv, i + 32);
+            list_load(i + 64, mv, moff);
+        }
+        if (DB && more) cp_async_wait<1>();
+        else cp_async_wait<0>();
         __syncwarp();
-        if (ehi >= e1) break;
+        window_pull<KIND, PACKED, L>(P, g, xs + buf * 32 * RW, vs, coff, 0u, cv, e, ehi, n_edges, n_upd, n_read);
+        __syncwarp();
+        if (!more) break;
+        if constexpr (!DB) rows_async(xs, nv, i + 32);
         e = ehi;
         i += 32;
+        if constexpr (DB) buf ^= 1;
+        cv = nv;
+        coff = noff;
+        nv = mv;
+        noff = moff;
     }
 }
 
@@ -1063,8 +1088,6 @@ __device__ __forceinline__ uint32_t first_entry(const BParams& P, uint32_t count
     return lo + 31 - __clz(__ballot_sync(FULL, le));
 }
 
-template <class L>  // 128 B rows (RW = 32): one window buffer, so 16 warps' buffers fit in shared memory
-constexpr bool xs_double() { return L::RW <= 16; }
 
 // S2 over the compacted list: the iteration's E list edges split evenly over all warps; a warp
 // slides 32-entry windows (a hub row is shared by as many warps and CTAs as needed).  Windows
