@@ -1775,9 +1775,12 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
         }
     }
     {   // phase-1 pull (relax_pull_all) over the kind's CG^R: iterations whose push would scan at
-        // least m_cg / CG_PULL_DIV edges (CG_PULL_DIV=0 disables it)
+        // least m_cg / CG_PULL_DIV edges (CG_PULL_DIV=0 disables it).  Default: REACH's bit lanes
+        // only — measured on C2 (profiles/r2_pull_experiments.txt): with 64 B value rows the
+        // segmented scan over 16 row words costs more than the atomics it saves (REACH 0.76 ->
+        // 0.69 ms; SSSP 2.53 -> 3.21 ms)
         const char* e = getenv("CG_PULL_DIV");
-        const uint32_t div = e ? (uint32_t)strtoul(e, nullptr, 10) : 2u;
+        const uint32_t div = e ? (uint32_t)strtoul(e, nullptr, 10) : (lw == 1 ? 2u : 0u);
         P.pl_thr = 0;
         if (c.two_phase && c.cg && div && c.cg->rcg_built && c.kind != CG_WCC) {
             const Core& C = *c.cg;
