@@ -14,6 +14,7 @@ import ncu_lines  # noqa: E402
 import ncu_summary  # noqa: E402
 
 KINDS = ("sssp", "sswp", "ssnp", "viterbi", "bfs", "reach")
+OUT = os.environ.get("NCU_OUT", os.path.join(ROOT, "profiles"))
 
 
 def num(v):
@@ -23,7 +24,7 @@ def num(v):
 def main(tag="r2"):
     out = {}
     for k in KINDS:
-        rep = os.path.join(ROOT, "gpurun_out", f"{tag}_ncu_{k}.ncu-rep")
+        rep = os.path.join(os.environ.get("NCU_DIR", os.path.join(ROOT, "gpurun_out")), f"{tag}_ncu_{k}.ncu-rep")
         if not os.path.exists(rep):
             continue
         rows = ncu_summary.raw(rep)
@@ -31,7 +32,8 @@ def main(tag="r2"):
             continue
         r = rows[0]
         unit_scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}
-        tscale = {"nsecond": 1e-6, "usecond": 1e-3, "msecond": 1.0, "second": 1e3}
+        tscale = {"nsecond": 1e-6, "usecond": 1e-3, "msecond": 1.0, "second": 1e3, "ns": 1e-6, "us": 1e-3, "ms": 1.0,
+                  "s": 1e3}
         rd = num(r["dram__bytes_read.sum"][0]) * unit_scale[r["dram__bytes_read.sum"][1]]
         wr = num(r["dram__bytes_write.sum"][0]) * unit_scale[r["dram__bytes_write.sum"][1]]
         ms = num(r["gpu__time_duration.sum"][0]) * tscale[r["gpu__time_duration.sum"][1]]
@@ -44,10 +46,10 @@ def main(tag="r2"):
             ncu_summary.main(rep)
             print("\nstall samples per source line:")
             ncu_lines.main(rep, 40)
-        with open(os.path.join(ROOT, "profiles", f"{tag}_ncu_{k}.txt"), "w") as f:
+        with open(os.path.join(OUT, f"{tag}_ncu_{k}.txt"), "w") as f:
             f.write(buf.getvalue())
         print(k, round(ms, 3), "ms", round((rd + wr) / 1e9, 3), "GB", round((rd + wr) / (ms / 1e3) / 1e9, 1), "GB/s")
-    path = os.path.join(ROOT, "profiles", "ncu_kinds.json")
+    path = os.path.join(OUT, "ncu_kinds.json")
     d = {}
     if os.path.exists(path):
         d = json.load(open(path))

@@ -6,7 +6,7 @@ tag=${1:-r2}
 mkdir -p gpurun_out
 for k in ${KINDS:-sssp sswp ssnp viterbi bfs reach}; do
   timeout 900 ncu --set full --nvtx --nvtx-include "prof/" --clock-control none --import-source on -f \
-    --kernel-name regex:"batch_kernel" -o gpurun_out/${tag}_ncu_${k} \
+    --kernel-name regex:"batch_kernel" -o ${NCU_DIR:-gpurun_out}/${tag}_ncu_${k} \
     python tools/profile_query.py --config c2 --kind $k --mode 2phase --batch 32 > gpurun_out/${tag}_ncu_${k}.log 2>&1
   tail -1 gpurun_out/${tag}_ncu_${k}.log
 done
