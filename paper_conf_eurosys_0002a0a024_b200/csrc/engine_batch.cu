@@ -30,9 +30,6 @@ namespace {
 
 using namespace kern;
 
-#ifndef CGB_STREAM
-#define CGB_STREAM 1  // S2 as one pipeline across windows (relax_stream); 0: per-window (relax_range)
-#endif
 #ifndef CGB_BT
 #define CGB_BT 512
 #endif
@@ -1163,214 +1160,6 @@ __device__ void relax_range(const BParams& P, const GraphView& g, uint32_t count
     }
 }
 
-// S2 as ONE software pipeline over the warp's whole edge range (round 2): the chunks of
-// consecutive 32-row windows flow through the same fetch (edge words) -> request (row gathers)
-// -> consume stages without draining at window boundaries.  relax_range's per-window pipeline
-// fill and drain cost about two memory latencies per window, which dominates when rows are short
-// (phase-1 CG rows average ~4 edges: ~4 chunks per window).  Up to three windows are live: each
-// has a context (per lane: its row's edge offset, address base and query mask) and an xs buffer
-// of source rows, copied (cp.async) when the fetch stage opens the window; a window's buffer is
-// reused after its last chunk has been consumed.  Entries that find no free window (windows
-// shorter than the pipeline) flow through empty.  Same per-chunk work as window_edges.
-template <int KIND, bool PACKED, class L>
-__device__ void relax_stream(const BParams& P, const GraphView& g, uint32_t count, uint32_t E, uint32_t e0, uint32_t e1,
-                             uint32_t* xs, uint32_t* vs, bool set_bits, bool fresh, uint32_t& n_edges,
-                             uint32_t& n_upd, uint32_t& n_read) {
-    constexpr int RW = L::RW;
-    using RC = RowCopy<L>;
-    constexpr int EA = (L::QPW == 2 && E_AHEAD == S_PIPE) ? 2 * S_PIPE : E_AHEAD;
-    constexpr int S = S_PIPE;
-    static_assert(EA % S == 0 && EA >= S, "E_AHEAD must be a multiple of S_PIPE");
-    constexpr uint32_t NONE = 0xffffffffu;
-    constexpr uint32_t WLAST = 4u, WFINAL = 8u;  // entry flags beside the window slot (bits 0-1)
-    const uint32_t lane = threadIdx.x & 31;
-    const uint32_t swz = RC::sw(lane);
-    if (e0 >= e1) return;
-
-    auto list_load = [&](uint32_t i0, uint32_t& v, uint32_t& off, uint32_t& mask) {
-        const uint32_t idx = i0 + lane;
-        v = 0;
-        off = E;
-        mask = 0;
-        if (idx < count) {
-            v = ld_cg(P.lv + idx);
-            off = ld_cg(P.lo + idx);
-            mask = ld_cg(P.lm + idx);
-        }
-    };
-    auto rows_async = [&](uint32_t* buf, uint32_t v, uint32_t i0) {  // the window's 32 source rows -> buf
-#pragma unroll
-        for (uint32_t r = 0; r < RC::C; ++r) {
-            const uint32_t f = r * 32 + lane, row = f / RC::C, c = f % RC::C;
-            const uint32_t vr = __shfl_sync(FULL, v, row);
-            if (i0 + row < count) RC::copy(buf + row * RW + c * RC::CW4, P.V + (size_t)vr * RW + c * RC::CW4, false);
-        }
-        cp_async_commit();
-    };
-
-    // window contexts, slots 0..2 (explicit registers: no dynamically indexed arrays)
-    uint32_t o0 = E, o1 = E, o2 = E, b0 = 0, b1 = 0, b2 = 0, m0 = 0, m1 = 0, m2 = 0;
-    uint32_t hi0 = 0, hi1 = 0, hi2 = 0;  // each live window's edge end (warp-uniform)
-    auto sel3 = [](uint32_t w, uint32_t a, uint32_t b, uint32_t c) { return w == 0 ? a : (w == 1 ? b : c); };
-
-    // list prefetch: pre1 = the next window to open (base ready), pre2 = the one after (loaded)
-    uint32_t i_open = first_entry(P, count, e0);  // list index of the next window to open
-    uint32_t p1v, p1o, p1m, p1b, p2v, p2o, p2m;
-    list_load(i_open, p1v, p1o, p1m);
-    p1b = (i_open + lane < count) ? __ldg(g.ptr + p1v) - p1o : 0u;
-    list_load(i_open + 32, p2v, p2o, p2m);
-    uint32_t f_lo = e0;       // first edge of the next window to open
-    bool all_open = false;    // every window of [e0, e1) has been opened
-
-    uint32_t fw = 0, fcs = 0, fhi = 0;  // fetch cursor: window slot, next chunk start, window end
-    bool fhave = false;                 // the fetch cursor is inside an open window
-    uint32_t nopen = 0;                 // windows opened so far; slot of window k = k % 3
-    uint32_t cw = 0;                    // windows fully consumed so far (a slot is free if < 3 live)
-
-    // open the next window into slot (nopen % 3): context from pre1, its rows copied, lists shifted
-    auto open_next = [&]() {
-        const uint32_t w = nopen % 3;
-        const uint32_t wend = (i_open + 32 < count) ? __shfl_sync(FULL, p2o, 0) : E;  // lo[i_open + 32]
-        const uint32_t hi = min(e1, wend);
-        if (w == 0) { o0 = p1o; b0 = p1b; m0 = p1m; hi0 = hi; }
-        else if (w == 1) { o1 = p1o; b1 = p1b; m1 = p1m; hi1 = hi; }
-        else { o2 = p1o; b2 = p1b; m2 = p1m; hi2 = hi; }
-        rows_async(xs + w * 32 * RW, p1v, i_open);
-        fw = w;
-        fcs = f_lo;
-        fhi = hi;
-        fhave = true;
-        ++nopen;
-        if (hi >= e1) {
-            all_open = true;
-        } else {
-            f_lo = hi;
-            i_open += 32;
-            p1v = p2v;
-            p1o = p2o;
-            p1m = p2m;
-            p1b = (i_open + lane < count) ? __ldg(g.ptr + p1v) - p1o : 0u;  // p2 was loaded a window ago
-            list_load(i_open + 32, p2v, p2o, p2m);
-        }
-    };
-
-    // fetch one pipeline entry: the next chunk's edge word (kout: its window row, NONE if none)
-    // and the entry's tag (window slot | WLAST | WFINAL, or NONE for an empty entry)
-    auto fetch = [&](EdgeWord<PACKED>& wd, uint32_t& kout, uint32_t& tag) {
-        kout = NONE;
-        tag = NONE;
-        if (!fhave) {
-            if (all_open || nopen - cw >= 3u) return;  // nothing left, or no free window slot yet
-            open_next();
-        }
-        const uint32_t cs = fcs, t = cs + lane;
-        const uint32_t off = sel3(fw, o0, o1, o2), base = sel3(fw, b0, b1, b2), mask = sel3(fw, m0, m1, m2);
-        const uint32_t below = __popc(__ballot_sync(FULL, off <= cs));  // >= 1: row 0 starts at or before cs
-        const uint32_t rel = off - cs;
-        const uint32_t starts = __reduce_or_sync(FULL, (rel - 1u < 31u) ? (1u << rel) : 0u);
-        const uint32_t kk = below - 1u + __popc(starts & ((2u << lane) - 1u));
-        const uint32_t mk = __shfl_sync(FULL, mask, kk);
-        const uint32_t a = __shfl_sync(FULL, base, kk) + t;
-        const bool ok = t < fhi && mk != 0u;
-        if (ok) wd.load(g, a);
-        kout = ok ? kk : NONE;
-        fcs = cs + 32;
-        tag = fw;
-        if (fcs >= fhi) {  // the window's last chunk
-            tag |= WLAST | (fhi >= e1 ? WFINAL : 0u);
-            fhave = false;
-        }
-    };
-
-    EdgeWord<PACKED> ew[EA];
-    uint32_t ek[EA], et[EA];
-    uint32_t sd[S], sw[S], sk[S], st[S];
-    auto request = [&](int slot, const EdgeWord<PACKED>& wd, uint32_t kk, uint32_t tag) {
-        sk[slot] = kk;
-        st[slot] = tag;
-        uint32_t dd = NONE;
-        if (kk != NONE) {
-            uint32_t d, w;
-            wd.decode(P.dbits, P.dmask, d, w);
-            sd[slot] = d;
-            sw[slot] = w;
-            dd = d;
-        }
-        if constexpr (RC::C > 1) {
-            constexpr uint32_t RPI = 32 / RC::C;
-            const uint32_t p = lane % RC::C;
-#pragma unroll
-            for (uint32_t i = 0; i < RC::C; ++i) {
-                const uint32_t r = i * RPI + lane / RC::C;
-                const uint32_t dr = __shfl_sync(FULL, dd, r);
-                if (dr != NONE)
-                    RC::copy(vs + (slot * 32 + r) * RW + RC::CW4 * (p ^ RC::sw(r)), P.V + (size_t)dr * RW + RC::CW4 * p,
-                             fresh);
-            }
-        } else if (dd != NONE) {
-            RC::copy(vs + (slot * 32 + lane) * RW, P.V + (size_t)dd * RW, fresh);
-        }
-        cp_async_commit();
-    };
-
-#pragma unroll
-    for (int s = 0; s < EA; ++s) fetch(ew[s], ek[s], et[s]);
-#pragma unroll
-    for (int s = 0; s < S - 1; ++s) {
-        request(s, ew[s], ek[s], et[s]);
-        fetch(ew[s], ek[s], et[s]);
-    }
-    for (;;) {
-#pragma unroll
-        for (int s = 0; s < EA; ++s) {
-            const int je = (s + S - 1) % EA;
-            const int jr = (s + S - 1) % S;
-            if constexpr (RC::C > 1) __syncwarp();
-            request(jr, ew[je], ek[je], et[je]);
-            fetch(ew[je], ek[je], et[je]);
-            cp_async_wait<S - 1>();
-            if constexpr (RC::C > 1) __syncwarp();
-            const int sr = s % S;
-            const uint32_t kk = sk[sr], tag = st[sr];
-            if (tag == NONE) continue;  // an empty entry
-            const uint32_t win = tag & 3u;
-            const uint32_t mk = __shfl_sync(FULL, sel3(win, m0, m1, m2), kk & 31u);
-            if (kk != NONE) {
-                ++n_read;
-                const uint32_t d = sd[sr];
-                const typename L::Arg w = L::arg(sw[sr]);
-                const uint32_t* rv = vs + (sr * 32 + lane) * RW;
-                const uint32_t* ru = xs + win * 32 * RW + kk * RW;
-                uint32_t* pv = P.V + (size_t)d * RW;
-                uint32_t changed = 0;
-#pragma unroll
-                for (int gi = 0; gi < RW / L::G; ++gi) {
-                    const uint32_t act = group_mask<L>(mk, gi);
-                    if (!act) continue;
-                    uint32_t uu[L::G], cc2[L::G];
-#pragma unroll
-                    for (int j = 0; j < L::G; ++j) {
-                        const uint32_t i = (uint32_t)(gi * L::G + j);
-                        uu[j] = ru[i];
-                        cc2[j] = rv[((i / RC::CW4) ^ swz) * RC::CW4 + i % RC::CW4];
-                    }
-                    changed |= L::relax(pv + gi * L::G, uu, cc2, w, act, n_edges, n_upd, P.err) << (gi * L::G * L::QPW);
-                }
-                if (changed) {
-                    red_or(P.M + d, changed);
-                    if (set_bits) red_or(P.bitmap + (d >> 5), 1u << (d & 31));
-                }
-            }
-            if (tag & WLAST) ++cw;  // the window's slot may be reopened (after the next __syncwarp)
-            if (tag & WFINAL) {
-                cp_async_wait<0>();
-                __syncwarp();
-                return;
-            }
-        }
-    }
-}
-
 // The iteration's E list edges over all warps: a static half split evenly (edge-balanced), then
 // — for iterations long enough to amortise a tile's list search — the rest in tiles taken from
 // a per-iteration counter, so warps slowed by contended EdgeFunctions (phase 1's hub rows) do
@@ -1390,12 +1179,7 @@ __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, ui
     const uint32_t T = dyn ? max(1024u, (uint32_t)((E - Es + NW - 1) / NW)) : 0u;
     uint32_t a = (uint32_t)((uint64_t)Es * gw / NW), b = (uint32_t)((uint64_t)Es * (gw + 1) / NW);
     for (;;) {  // one call site: the range body is inlined once
-#if CGB_STREAM
-        if constexpr (L::RW <= 16)
-            relax_stream<KIND, PACKED, L>(P, g, count, E, a, b, xs, vs, set_bits, fresh, n_edges, n_upd, n_read);
-        else
-#endif
-            relax_range<KIND, PACKED, L>(P, g, count, E, a, b, xs, vs, set_bits, fresh, n_edges, n_upd, n_read);
+        relax_range<KIND, PACKED, L>(P, g, count, E, a, b, xs, vs, set_bits, fresh, n_edges, n_upd, n_read);
         if (!dyn) break;
         unsigned long long t = 0;
         if (lane == 0) t = atomicAdd(tiles, 1ull);
@@ -1645,8 +1429,6 @@ __device__ void transpose_narrow(const BParams& P, int q0, int nq, uint32_t* xs)
 
 template <class L>  // per warp, 16 B aligned: one or two 32-row windows (S2) or the padded transpose tile
 constexpr uint32_t xs_words() {
-    if constexpr (CGB_STREAM && L::RW <= 16) return 3 * 32 * L::RW > 32 * (L::RW + 1) + 3 ? 3 * 32 * L::RW
-                                                                                          : ((32 * (L::RW + 1) + 3) & ~3u);
     return (xs_double<L>() ? 2 : 1) * 32 * L::RW > ((32 * (L::RW + 1) + 3) & ~3u) ? (xs_double<L>() ? 2 : 1) * 32 * L::RW
                                                                                  : ((32 * (L::RW + 1) + 3) & ~3u);
 }
