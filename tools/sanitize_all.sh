@@ -5,7 +5,7 @@ mkdir -p gpurun_out
 for tool in memcheck racecheck synccheck initcheck; do
   extra=""
   [ $tool = initcheck ] && extra="--track-unused-memory no"
-  timeout 2400 compute-sanitizer --tool $tool $extra --kernel-name regex:'batch_kernel|query_kernel|k_' \
+  timeout 2400 compute-sanitizer --tool $tool $extra --kernel-name kns=cgb \
     --print-limit 50 python tools/sanitize_run.py > gpurun_out/sanitize_$tool.txt 2>&1
   echo "$tool rc=$? $(tail -2 gpurun_out/sanitize_$tool.txt | tr '\n' ' ')"
 done
