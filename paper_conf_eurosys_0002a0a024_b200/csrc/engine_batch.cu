@@ -1175,8 +1175,14 @@ __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, ui
     const uint32_t gw = blockIdx.x * BW + (threadIdx.x >> 5);
     const uint64_t NW = (uint64_t)gridDim.x * BW;
     const bool dyn = tiles != nullptr && (uint64_t)E >= NW * CGB_DYN_MIN;
-    const uint32_t Es = dyn ? E / 2 : E;
-    const uint32_t T = dyn ? max(1024u, (uint32_t)((E - Es + NW - 1) / NW)) : 0u;
+#ifndef CGB_DYN_STATIC
+#define CGB_DYN_STATIC 2  // 1 / (static share of a dynamic iteration's edges)
+#endif
+#ifndef CGB_DYN_TPW
+#define CGB_DYN_TPW 1     // dynamic tiles per warp
+#endif
+    const uint32_t Es = dyn ? E / CGB_DYN_STATIC : E;
+    const uint32_t T = dyn ? max(1024u / CGB_DYN_TPW, (uint32_t)((E - Es + NW * CGB_DYN_TPW - 1) / (NW * CGB_DYN_TPW))) : 0u;
     uint32_t a = (uint32_t)((uint64_t)Es * gw / NW), b = (uint32_t)((uint64_t)Es * (gw + 1) / NW);
     for (;;) {  // one call site: the range body is inlined once
         relax_range<KIND, PACKED, L>(P, g, count, E, a, b, xs, vs, set_bits, fresh, n_edges, n_upd, n_read);
