@@ -1179,7 +1179,7 @@ __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, ui
 #define CGB_DYN_STATIC 2  // 1 / (static share of a dynamic iteration's edges)
 #endif
 #ifndef CGB_DYN_TPW
-#define CGB_DYN_TPW 1     // dynamic tiles per warp
+#define CGB_DYN_TPW 4     // dynamic tiles per warp (measured on C2: 1 -> 11.79 K q/s, 2 -> 11.86 K (static 1/4), 4 -> 12.24 K)
 #endif
     const uint32_t Es = dyn ? E / CGB_DYN_STATIC : E;
     const uint32_t T = dyn ? max(1024u / CGB_DYN_TPW, (uint32_t)((E - Es + NW * CGB_DYN_TPW - 1) / (NW * CGB_DYN_TPW))) : 0u;
