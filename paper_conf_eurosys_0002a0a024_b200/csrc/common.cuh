@@ -106,13 +106,6 @@ __device__ __forceinline__ uint32_t ld_stream(const uint32_t* p) {
                  : "l"(p), "l"(policy_evict_first()));
     return v;
 }
-__device__ __forceinline__ uint4 ld_stream4(const uint4* p) {
-    uint4 v;
-    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
-                 : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
-                 : "l"(p), "l"(policy_evict_first()));
-    return v;
-}
 __device__ __forceinline__ uint2 ld_stream2(const uint2* p) {
     uint2 v;
     asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v2.u32 {%0,%1}, [%2], %3;"
@@ -120,7 +113,6 @@ __device__ __forceinline__ uint2 ld_stream2(const uint2* p) {
                  : "l"(p), "l"(policy_evict_first()));
     return v;
 }
-__device__ __forceinline__ uint32_t ld_ro(const uint32_t* p) { return __ldg(p); }
 
 __device__ __forceinline__ void red_or(uint32_t* p, uint32_t v) {
     asm volatile("red.relaxed.gpu.global.or.b32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
@@ -133,33 +125,8 @@ __device__ __forceinline__ void red_max(uint32_t* p, uint32_t v) {
     asm volatile("red.relaxed.gpu.global.max.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 
-// ---------------------------------------------------------------- TMA (bulk async copy) + mbarrier
+// ---------------------------------------------------------------- shared-memory address
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
-__device__ __forceinline__ void mbar_init(unsigned long long* bar, uint32_t count) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void fence_mbar_init() { asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory"); }
-__device__ __forceinline__ void mbar_expect_tx(unsigned long long* bar, uint32_t bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(unsigned long long* bar, uint32_t parity) {
-    asm volatile(
-        "{\n\t.reg .pred p;\n"
-        "WAIT_%=:\n\t"
-        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
-        "@!p bra WAIT_%=;\n}" ::"r"(smem_u32(bar)),
-        "r"(parity)
-        : "memory");
-}
-// 1D bulk copy global -> shared (TMA engine), completion counted on `bar`, evict-first in L2
-__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, unsigned long long* bar) {
-    asm volatile(
-        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;" ::"r"(
-            smem_u32(dst)),
-        "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(policy_evict_first())
-        : "memory");
-}
-
 __device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31u; }
 
 // ---------------------------------------------------------------- cp.async (LDGSTS): 16 B global -> shared

@@ -527,6 +527,9 @@ __device__ void compact_bits(const BParams& P, const GraphView& g, unsigned long
     }
 }
 
+#ifndef CGB_S1_SPARSE
+#define CGB_S1_SPARSE 1  // S1 reads row bounds only for vertices with a nonzero mask
+#endif
 // S1 for large frontiers held as query masks M (F_MASKS, and F_IMPACTED / F_UNCERT after their
 // mark pass): no bitmap.  A warp issues the masks and row offsets of 16 bitmap words (512
 // vertices) at once — one memory round trip instead of a dependent degree fetch per active word.
@@ -534,6 +537,26 @@ __device__ __forceinline__ void span_loads(const BParams& P, const GraphView& g,
                                            uint32_t (&mv)[16], uint32_t (&dg)[16]) {
     const uint32_t lane = threadIdx.x & 31;
     uint32_t pv[16];
+#if CGB_S1_SPARSE
+    // masks first, then the row bounds of the active vertices only: sparse frontiers (most
+    // iterations) read M alone instead of M + two offset arrays
+#pragma unroll
+    for (int j = 0; j < 16; ++j) {
+        const uint32_t wj = g0 + h * 16 + j;
+        const uint32_t v = wj * 32 + lane;
+        mv[j] = (wj < w1 && v < P.n) ? ld_cg(P.M + v) : 0u;
+    }
+    const uint32_t* pe = g.end ? g.end : g.ptr + 1;
+#pragma unroll
+    for (int j = 0; j < 16; ++j) {
+        const uint32_t v = (g0 + h * 16 + j) * 32 + lane;
+        pv[j] = mv[j] ? __ldg(g.ptr + v) : 0u;
+        dg[j] = mv[j] ? __ldg(pe + v) : 0u;
+    }
+#pragma unroll
+    for (int j = 0; j < 16; ++j) dg[j] -= pv[j];
+    return;
+#endif
     if (g.end) {  // split rows: [ptr[v], end[v])
 #pragma unroll
         for (int j = 0; j < 16; ++j) {
@@ -686,6 +709,14 @@ template <class L> struct RowCopy {
     }
 };
 
+// edge-word lead over the row requests (chunks): binary16 rows (the cheapest relax per edge) keep
+// the edge stream 2 x S_PIPE chunks ahead by default; the u32 rows' heavier relax needs the registers
+#ifndef CGB_EA16
+#define CGB_EA16 (2 * CGB_STAGES)
+#endif
+template <class L>
+constexpr int ea_lead() { return (L::QPW == 2 && E_AHEAD == S_PIPE) ? CGB_EA16 : E_AHEAD; }
+
 // The edges [e, ehi) of one 32-row window: lane r of the window holds row r's first edge index
 // `off`, its address base (edge address = base + edge index) and its query mask; the rows'
 // values are in xs (r * RW + word).  Lane L takes edge L of each 32-edge chunk for all Q queries.
@@ -698,9 +729,7 @@ __device__ __forceinline__ void window_edges(const BParams& P, const GraphView& 
                                              uint32_t off, uint32_t base, uint32_t mask, uint32_t e, uint32_t ehi,
                                              bool set_bits, bool fresh, uint32_t& n_edges, uint32_t& n_upd,
                                              uint32_t& n_read) {
-    // binary16 rows (the cheapest relax per edge) keep the edge stream 4 chunks ahead; the u32
-    // rows' heavier relax needs the registers (measured: Viterbi 16 % slower with 4)
-    constexpr int EA = (L::QPW == 2 && E_AHEAD == S_PIPE) ? 2 * S_PIPE : E_AHEAD;
+    constexpr int EA = ea_lead<L>();
     constexpr int S = S_PIPE, RW = L::RW;
     static_assert(EA % S == 0 && EA >= S, "E_AHEAD must be a multiple of S_PIPE");
     using RC = RowCopy<L>;
@@ -712,7 +741,13 @@ __device__ __forceinline__ void window_edges(const BParams& P, const GraphView& 
 
     EdgeWord<PACKED> ew[EA];       // fetched edge words (slot = chunk % EA)
     uint32_t ek[EA];               // their window row (NONE: no edge / inactive row)
-    uint32_t sd[S], sw[S], sk[S];  // requested chunks (slot = chunk % S): destination, weight, window row
+    // requested chunks (slot = chunk % S): destination, weight, window row of each lane's edge —
+    // kept in the warp's shared metadata ring (lane-private words), not in registers, so the
+    // row pipeline can be deeper without spilling
+    uint32_t* const mt = vs + S * 32 * RW;
+    auto sd = [&](int slot) -> uint32_t& { return mt[(3 * slot + 0) * 32 + lane]; };
+    auto sw = [&](int slot) -> uint32_t& { return mt[(3 * slot + 1) * 32 + lane]; };
+    auto sk = [&](int slot) -> uint32_t& { return mt[(3 * slot + 2) * 32 + lane]; };
 
     // the window row of each lane's edge t = cs + lane: rows starting at or before cs (one
     // ballot) plus the rows starting in (cs, t] (one warp OR of start bits) — no dependent
@@ -734,13 +769,13 @@ __device__ __forceinline__ void window_edges(const BParams& P, const GraphView& 
     // contiguous 16 B pieces instead of 32 scattered lines (C times fewer L1 tag lookups per
     // chunk).  The slot is shared across lanes, so the caller brackets it with __syncwarp().
     auto request = [&](int slot, const EdgeWord<PACKED>& wd, uint32_t kk) {
-        sk[slot] = kk;
+        sk(slot) = kk;
         uint32_t dd = NONE;
         if (kk != NONE) {
             uint32_t d, w;
             wd.decode(P.dbits, P.dmask, d, w);
-            sd[slot] = d;
-            sw[slot] = w;
+            sd(slot) = d;
+            sw(slot) = w;
             dd = d;
         }
         if constexpr (RC::C > 1) {
@@ -785,12 +820,12 @@ __device__ __forceinline__ void window_edges(const BParams& P, const GraphView& 
             cp_async_wait<S - 1>();  // chunk cc's row pieces this lane copied have landed
             if constexpr (RC::C > 1) __syncwarp();  // ... and those the other lanes copied
             const int sr = s % S;    // chunk cc's row slot
-            const uint32_t kk = sk[sr];
+            const uint32_t kk = sk(sr);
             const uint32_t mk = __shfl_sync(FULL, mask, kk & 31u);
             if (kk == NONE) continue;
             ++n_read;
-            const uint32_t d = sd[sr];
-            const typename L::Arg w = L::arg(sw[sr]);         // per edge, shared by the row's queries
+            const uint32_t d = sd(sr);
+            const typename L::Arg w = L::arg(sw(sr));         // per edge, shared by the row's queries
             const uint32_t* rv = vs + (sr * 32 + lane) * RW;  // v's row (swizzled copies)
             const uint32_t* ru = xs + kk * RW;               // u's row
             uint32_t* pv = P.V + (size_t)d * RW;
@@ -1088,6 +1123,37 @@ __device__ __forceinline__ uint32_t first_entry(const BParams& P, uint32_t count
     return lo + 31 - __clz(__ballot_sync(FULL, le));
 }
 
+// S2's work split in COST units: list entry i costs ALPHA (its window slot, row offsets, source-row
+// copy) plus one per edge, i.e. entry i spans costs [lo[i] + ALPHA i, lo[i+1] + ALPHA (i+1)), its
+// ALPHA slot first.  cost_edge(c) = the edge at cost c (the entry's first edge while c is inside
+// its slot): monotone, so consecutive warps' cost ranges map to disjoint, covering edge ranges.
+// With ALPHA = 0 a cost is an edge index (a pure edge-balanced split).
+#ifndef CGB_ALPHA
+#define CGB_ALPHA 0u
+#endif
+__device__ __forceinline__ uint32_t cost_edge(const BParams& P, uint32_t count, uint32_t E, uint64_t c) {
+    constexpr uint64_t A = CGB_ALPHA;
+    if (A == 0) return (uint32_t)min(c, (uint64_t)E);
+    if (c >= (uint64_t)E + A * count) return E;
+    const uint32_t lane = threadIdx.x & 31;
+    uint32_t lo = 0, hi = count;
+    while (hi - lo > 32) {
+        const uint32_t step = (hi - lo + 31) / 32;
+        const uint32_t p = lo + lane * step;
+        const bool le = p < hi && ld_cg(P.lo + p) + A * p <= c;
+        const uint32_t k = 31 - __clz(__ballot_sync(FULL, le));
+        const uint32_t nlo = lo + k * step;
+        hi = min(hi, nlo + step);
+        lo = nlo;
+    }
+    const uint32_t p = lo + lane;
+    const uint32_t x = p < hi ? ld_cg(P.lo + p) : 0u;
+    const bool le = p < hi && x + A * p <= c;
+    const uint32_t i = lo + 31 - __clz(__ballot_sync(FULL, le));
+    const uint64_t ci = __shfl_sync(FULL, x, i - lo);
+    return (uint32_t)(ci + (c > ci + A * i + A ? c - ci - A * i - A : 0u));
+}
+
 
 // S2 over the compacted list: the iteration's E list edges split evenly over all warps; a warp
 // slides 32-entry windows (a hub row is shared by as many warps and CTAs as needed).  Windows
@@ -1181,19 +1247,20 @@ __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, ui
 #ifndef CGB_DYN_TPW
 #define CGB_DYN_TPW 4     // dynamic tiles per warp (measured on C2: 1 -> 11.79 K q/s, 2 -> 11.86 K (static 1/4), 4 -> 12.24 K)
 #endif
-    const uint32_t Es = dyn ? E / CGB_DYN_STATIC : E;
-    const uint32_t T = dyn ? max(1024u / CGB_DYN_TPW, (uint32_t)((E - Es + NW * CGB_DYN_TPW - 1) / (NW * CGB_DYN_TPW))) : 0u;
-    uint32_t a = (uint32_t)((uint64_t)Es * gw / NW), b = (uint32_t)((uint64_t)Es * (gw + 1) / NW);
+    const uint64_t C = (uint64_t)E + (uint64_t)CGB_ALPHA * count;  // total cost (= E for ALPHA 0)
+    const uint64_t Cs = dyn ? C / CGB_DYN_STATIC : C;
+    const uint64_t T = dyn ? max((uint64_t)(1024u / CGB_DYN_TPW), (C - Cs + NW * CGB_DYN_TPW - 1) / (NW * CGB_DYN_TPW)) : 0u;
+    uint64_t a = Cs * gw / NW, b = Cs * (gw + 1) / NW;
     for (;;) {  // one call site: the range body is inlined once
-        relax_range<KIND, PACKED, L>(P, g, count, E, a, b, xs, vs, set_bits, fresh, n_edges, n_upd, n_read);
+        relax_range<KIND, PACKED, L>(P, g, count, E, cost_edge(P, count, E, a), cost_edge(P, count, E, b), xs, vs,
+                                     set_bits, fresh, n_edges, n_upd, n_read);
         if (!dyn) break;
         unsigned long long t = 0;
         if (lane == 0) t = atomicAdd(tiles, 1ull);
         t = __shfl_sync(FULL, t, 0);
-        const uint64_t a64 = Es + t * T;
-        if (a64 >= E) break;
-        a = (uint32_t)a64;
-        b = (uint32_t)(a64 + T < E ? a64 + T : E);
+        a = Cs + t * T;
+        if (a >= C) break;
+        b = a + T < C ? a + T : C;
     }
 }
 
@@ -1439,10 +1506,10 @@ constexpr uint32_t xs_words() {
                                                                                  : ((32 * (L::RW + 1) + 3) & ~3u);
 }
 template <class L>
-constexpr uint32_t vs_words() { return S_PIPE * 32 * L::RW; }
+constexpr uint32_t vs_words() { return S_PIPE * 32 * L::RW + 3 * S_PIPE * 32; }  // row ring + metadata ring
 
 template <int KIND, bool PACKED, class L>
-__global__ void __launch_bounds__(BT, 512 / BT) batch_kernel(BParams P) {
+__global__ void __launch_bounds__(BT, BT <= 512 ? 512 / BT : 1) batch_kernel(BParams P) {
     constexpr int Q = L::Q, RW = L::RW;
     __shared__ uint32_t sm_cnt[2 * BW + 2];
     __shared__ unsigned long long sm_red[BW];

@@ -105,6 +105,9 @@ __device__ __forceinline__ void report_sticky(uint32_t* err_map, uint32_t e) {
 }
 
 // ------------------------------------------------------------------ grid barrier
+#ifndef CGB_BAR_SLEEP
+#define CGB_BAR_SLEEP 32  // ns between polls of the arrival counter (0: spin)
+#endif
 __device__ __forceinline__ void grid_sync(unsigned long long* bar, unsigned long long& epoch) {
     __syncthreads();
     ++epoch;
@@ -115,7 +118,9 @@ __device__ __forceinline__ void grid_sync(unsigned long long* bar, unsigned long
         for (;;) {  // relaxed polling: no per-poll L1 invalidation
             asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(cur) : "l"(bar) : "memory");
             if (cur >= target) break;
-            __nanosleep(32);
+#if CGB_BAR_SLEEP
+            __nanosleep(CGB_BAR_SLEEP);
+#endif
         }
         asm volatile("fence.acq_rel.gpu;" ::: "memory");
     }
