@@ -1123,38 +1123,6 @@ __device__ __forceinline__ uint32_t first_entry(const BParams& P, uint32_t count
     return lo + 31 - __clz(__ballot_sync(FULL, le));
 }
 
-// S2's work split in COST units: list entry i costs ALPHA (its window slot, row offsets, source-row
-// copy) plus one per edge, i.e. entry i spans costs [lo[i] + ALPHA i, lo[i+1] + ALPHA (i+1)), its
-// ALPHA slot first.  cost_edge(c) = the edge at cost c (the entry's first edge while c is inside
-// its slot): monotone, so consecutive warps' cost ranges map to disjoint, covering edge ranges.
-// With ALPHA = 0 a cost is an edge index (a pure edge-balanced split).
-#ifndef CGB_ALPHA
-#define CGB_ALPHA 0u
-#endif
-__device__ __forceinline__ uint32_t cost_edge(const BParams& P, uint32_t count, uint32_t E, uint64_t c) {
-    constexpr uint64_t A = CGB_ALPHA;
-    if (A == 0) return (uint32_t)min(c, (uint64_t)E);
-    if (c >= (uint64_t)E + A * count) return E;
-    const uint32_t lane = threadIdx.x & 31;
-    uint32_t lo = 0, hi = count;
-    while (hi - lo > 32) {
-        const uint32_t step = (hi - lo + 31) / 32;
-        const uint32_t p = lo + lane * step;
-        const bool le = p < hi && ld_cg(P.lo + p) + A * p <= c;
-        const uint32_t k = 31 - __clz(__ballot_sync(FULL, le));
-        const uint32_t nlo = lo + k * step;
-        hi = min(hi, nlo + step);
-        lo = nlo;
-    }
-    const uint32_t p = lo + lane;
-    const uint32_t x = p < hi ? ld_cg(P.lo + p) : 0u;
-    const bool le = p < hi && x + A * p <= c;
-    const uint32_t i = lo + 31 - __clz(__ballot_sync(FULL, le));
-    const uint64_t ci = __shfl_sync(FULL, x, i - lo);
-    return (uint32_t)(ci + (c > ci + A * i + A ? c - ci - A * i - A : 0u));
-}
-
-
 // S2 over the compacted list: the iteration's E list edges split evenly over all warps; a warp
 // slides 32-entry windows (a hub row is shared by as many warps and CTAs as needed).  Windows
 // are prefetched one ahead: while window i's edges run, window i+1's source rows are already
@@ -1247,20 +1215,19 @@ __device__ void relax_b(const BParams& P, const GraphView& g, uint32_t count, ui
 #ifndef CGB_DYN_TPW
 #define CGB_DYN_TPW 4     // dynamic tiles per warp (measured on C2: 1 -> 11.79 K q/s, 2 -> 11.86 K (static 1/4), 4 -> 12.24 K)
 #endif
-    const uint64_t C = (uint64_t)E + (uint64_t)CGB_ALPHA * count;  // total cost (= E for ALPHA 0)
-    const uint64_t Cs = dyn ? C / CGB_DYN_STATIC : C;
-    const uint64_t T = dyn ? max((uint64_t)(1024u / CGB_DYN_TPW), (C - Cs + NW * CGB_DYN_TPW - 1) / (NW * CGB_DYN_TPW)) : 0u;
-    uint64_t a = Cs * gw / NW, b = Cs * (gw + 1) / NW;
+    const uint32_t Es = dyn ? E / CGB_DYN_STATIC : E;
+    const uint32_t T = dyn ? max(1024u / CGB_DYN_TPW, (uint32_t)((E - Es + NW * CGB_DYN_TPW - 1) / (NW * CGB_DYN_TPW))) : 0u;
+    uint32_t a = (uint32_t)((uint64_t)Es * gw / NW), b = (uint32_t)((uint64_t)Es * (gw + 1) / NW);
     for (;;) {  // one call site: the range body is inlined once
-        relax_range<KIND, PACKED, L>(P, g, count, E, cost_edge(P, count, E, a), cost_edge(P, count, E, b), xs, vs,
-                                     set_bits, fresh, n_edges, n_upd, n_read);
+        relax_range<KIND, PACKED, L>(P, g, count, E, a, b, xs, vs, set_bits, fresh, n_edges, n_upd, n_read);
         if (!dyn) break;
         unsigned long long t = 0;
         if (lane == 0) t = atomicAdd(tiles, 1ull);
         t = __shfl_sync(FULL, t, 0);
-        a = Cs + t * T;
-        if (a >= C) break;
-        b = a + T < C ? a + T : C;
+        const uint64_t a64 = Es + t * T;
+        if (a64 >= E) break;
+        a = (uint32_t)a64;
+        b = (uint32_t)(a64 + T < E ? a64 + T : E);
     }
 }
 
@@ -1733,13 +1700,17 @@ __global__ void __launch_bounds__(BT, BT <= 512 ? 512 / BT : 1) batch_kernel(BPa
 template <int KIND, bool PACKED, int LW>
 void launch_b(const BParams& P, int sms, cudaStream_t s) {
     using L = typename LanesOf<LW, KIND>::T;
-    const size_t smem = ((size_t)BW * (xs_words<L>() + vs_words<L>()) + (size_t)L::Q * 2 * 64) * sizeof(uint32_t);
+    // the certificates' source hub values (sh) only when the call uses them: shared memory not
+    // allocated stays L1
+    const size_t base = (size_t)BW * (xs_words<L>() + vs_words<L>()) * sizeof(uint32_t);
+    const size_t smax = base + (size_t)L::Q * 2 * 64 * sizeof(uint32_t);
+    const size_t smem = P.HB ? smax : base;
     static int bps = 0;
     if (!bps) {
-        if (smem > 48 * 1024)
+        if (smax > 48 * 1024)
             CGB_CUDA(cudaFuncSetAttribute(batch_kernel<KIND, PACKED, L>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                          (int)smem));
-        CGB_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, batch_kernel<KIND, PACKED, L>, BT, smem));
+                                          (int)smax));
+        CGB_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, batch_kernel<KIND, PACKED, L>, BT, smax));
         CGB_CHECK(bps > 0, CG_EUNSUPPORTED, "batch kernel cannot be resident");
     }
     void* args[] = {(void*)&P};
