@@ -709,6 +709,14 @@ template <class L> struct RowCopy {
     }
 };
 
+#ifndef CGB_EDGE_SMEM
+#define CGB_EDGE_SMEM 2  // S2's edge words through a shared-memory ring (window_edges_sm): 0 never, 1 every
+                         // lane type, 2 one-word rows only (REACH bits, WCC labels; measured on C2: REACH
+                         // FULL 1.82 -> 1.54 ms, WCC 1.84 -> 1.53 ms; 64 B rows 2-5 % slower, and slower
+                         // still with a deeper row pipeline: profiles/r2_s2_experiments.txt)
+#endif
+template <class L>
+constexpr bool edge_smem() { return CGB_EDGE_SMEM == 1 || (CGB_EDGE_SMEM == 2 && L::RW == 1); }
 // edge-word lead over the row requests (chunks): binary16 rows (the cheapest relax per edge) keep
 // the edge stream 2 x S_PIPE chunks ahead by default; the u32 rows' heavier relax needs the registers
 #ifndef CGB_EA16
@@ -847,6 +855,121 @@ __device__ __forceinline__ void window_edges(const BParams& P, const GraphView& 
                 red_or(P.M + d, changed);                                 // v active for those queries
                 if (set_bits) red_or(P.bitmap + (d >> 5), 1u << (d & 31));  // union frontier bit
             }
+        }
+    }
+    cp_async_wait<0>();
+}
+
+// window_edges with the edge stream in shared memory as well: edge words are copied (cp.async, 4 or
+// 8 B per lane) into a per-warp ring LE = S_PIPE chunks ahead of the row requests, their window rows
+// into a lane-private ring beside it — no pipeline state in registers, so the row pipeline can be
+// deeper.  One cp.async group per chunk: {rows of chunk c + S - 1, edge words of chunk c + 2S - 1}.
+template <int KIND, bool PACKED, class L>
+__device__ __forceinline__ void window_edges_sm(const BParams& P, const GraphView& g, const uint32_t* xs,
+                                                uint32_t* vs, uint32_t off, uint32_t base, uint32_t mask, uint32_t e,
+                                                uint32_t ehi, bool set_bits, bool fresh, uint32_t& n_edges,
+                                                uint32_t& n_upd, uint32_t& n_read) {
+    constexpr uint32_t S = S_PIPE, LE = S_PIPE, NE = 2 * S_PIPE, RW = L::RW, EWW = PACKED ? 1 : 2;
+    using RC = RowCopy<L>;
+    constexpr uint32_t NONE = 0xffffffffu;
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t swz = RC::sw(lane);
+    if (e >= ehi) return;
+    const uint32_t nch = (ehi - e + 31) >> 5;
+    uint32_t* const mt = vs + S * 32 * RW;   // [S][3][32]: destination, weight, window row
+    uint32_t* const er = mt + 3 * S * 32;    // [NE][32][EWW]: edge words
+    uint32_t* const kr = er + NE * 32 * EWW; // [NE][32]: their window rows
+    auto fetch = [&](uint32_t c) {
+        const uint32_t slot = c % NE;
+        const uint32_t cs = e + c * 32, t = cs + lane;
+        const uint32_t below = __popc(__ballot_sync(FULL, off <= cs));
+        const uint32_t rel = off - cs;
+        const uint32_t starts = __reduce_or_sync(FULL, (rel - 1u < 31u) ? (1u << rel) : 0u);
+        const uint32_t kk = below - 1u + __popc(starts & ((2u << lane) - 1u));
+        const uint32_t mk = __shfl_sync(FULL, mask, kk);
+        const uint32_t a = __shfl_sync(FULL, base, kk) + t;
+        const bool ok = t < ehi && mk != 0u;
+        if (ok) {
+            if constexpr (PACKED)
+                asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(smem_u32(er + slot * 32 + lane)),
+                             "l"(g.adj + a) : "memory");
+            else
+                asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(smem_u32(er + (slot * 32 + lane) * 2)),
+                             "l"(g.adjw + a) : "memory");
+        }
+        kr[slot * 32 + lane] = ok ? kk : NONE;
+    };
+    auto request = [&](uint32_t c) {  // chunk c's edge word has landed (lane-private)
+        const uint32_t es = c % NE, rs = c % S;
+        const uint32_t kk = kr[es * 32 + lane];
+        mt[(3 * rs + 2) * 32 + lane] = kk;
+        uint32_t dd = NONE;
+        if (kk != NONE) {
+            EdgeWord<PACKED> wd;
+            if constexpr (PACKED) wd.x = er[es * 32 + lane];
+            else wd.x = *reinterpret_cast<const uint2*>(er + (es * 32 + lane) * 2);
+            uint32_t d, w;
+            wd.decode(P.dbits, P.dmask, d, w);
+            mt[(3 * rs + 0) * 32 + lane] = d;
+            mt[(3 * rs + 1) * 32 + lane] = w;
+            dd = d;
+        }
+        if constexpr (RC::C > 1) {
+            constexpr uint32_t RPI = 32 / RC::C;
+            const uint32_t p = lane % RC::C;
+#pragma unroll
+            for (uint32_t i = 0; i < RC::C; ++i) {
+                const uint32_t r = i * RPI + lane / RC::C;
+                const uint32_t dr = __shfl_sync(FULL, dd, r);
+                if (dr != NONE)
+                    RC::copy(vs + (rs * 32 + r) * RW + RC::CW4 * (p ^ RC::sw(r)), P.V + (size_t)dr * RW + RC::CW4 * p,
+                             fresh);
+            }
+        } else if (dd != NONE) {
+            RC::copy(vs + (rs * 32 + lane) * RW, P.V + (size_t)dd * RW, fresh);
+        }
+    };
+    for (uint32_t c = 0; c < S - 1 + LE && c < nch; ++c) fetch(c);
+    cp_async_commit();
+    cp_async_wait<0>();
+    for (uint32_t c = 0; c < S - 1; ++c) {
+        if (c < nch) request(c);
+        cp_async_commit();
+    }
+    for (uint32_t cc = 0; cc < nch; ++cc) {
+        if constexpr (RC::C > 1) __syncwarp();  // every lane is done with row slot (cc - 1) % S
+        if (cc + S - 1 < nch) request(cc + S - 1);
+        if (cc + S - 1 + LE < nch) fetch(cc + S - 1 + LE);
+        cp_async_commit();
+        cp_async_wait<S - 1>();                 // chunk cc's rows (and chunk cc + S's edge words) landed
+        if constexpr (RC::C > 1) __syncwarp();
+        const uint32_t sr = cc % S;
+        const uint32_t kk = mt[(3 * sr + 2) * 32 + lane];
+        const uint32_t mk = __shfl_sync(FULL, mask, kk & 31u);
+        if (kk == NONE) continue;
+        ++n_read;
+        const uint32_t d = mt[(3 * sr + 0) * 32 + lane];
+        const typename L::Arg w = L::arg(mt[(3 * sr + 1) * 32 + lane]);
+        const uint32_t* rv = vs + (sr * 32 + lane) * RW;
+        const uint32_t* ru = xs + kk * RW;
+        uint32_t* pv = P.V + (size_t)d * RW;
+        uint32_t changed = 0;
+#pragma unroll
+        for (int gi = 0; gi < (int)RW / L::G; ++gi) {
+            const uint32_t act = group_mask<L>(mk, gi);
+            if (!act) continue;
+            uint32_t uu[L::G], cc2[L::G];
+#pragma unroll
+            for (int j = 0; j < L::G; ++j) {
+                const uint32_t i = (uint32_t)(gi * L::G + j);
+                uu[j] = ru[i];
+                cc2[j] = rv[((i / RC::CW4) ^ swz) * RC::CW4 + i % RC::CW4];
+            }
+            changed |= L::relax(pv + gi * L::G, uu, cc2, w, act, n_edges, n_upd, P.err) << (gi * L::G * L::QPW);
+        }
+        if (changed) {
+            red_or(P.M + d, changed);
+            if (set_bits) red_or(P.bitmap + (d >> 5), 1u << (d & 31));
         }
     }
     cp_async_wait<0>();
@@ -1176,8 +1299,12 @@ __device__ void relax_range(const BParams& P, const GraphView& g, uint32_t count
         if (DB && more) cp_async_wait<1>();  // this window's rows (the next window's may still fly)
         else cp_async_wait<0>();
         __syncwarp();
-        window_edges<KIND, PACKED, L>(P, g, xs + buf * 32 * RW, vs, coff, cbase, cmask, e, ehi, set_bits, fresh,
-                                      n_edges, n_upd, n_read);
+        if constexpr (edge_smem<L>())
+            window_edges_sm<KIND, PACKED, L>(P, g, xs + buf * 32 * RW, vs, coff, cbase, cmask, e, ehi, set_bits, fresh,
+                                             n_edges, n_upd, n_read);
+        else
+            window_edges<KIND, PACKED, L>(P, g, xs + buf * 32 * RW, vs, coff, cbase, cmask, e, ehi, set_bits, fresh,
+                                          n_edges, n_upd, n_read);
         __syncwarp();  // every lane is done with this window's rows before they are overwritten
         if (!more) break;
         if constexpr (!DB) rows_async(xs, nv, i + 32);
@@ -1473,7 +1600,9 @@ constexpr uint32_t xs_words() {
                                                                                  : ((32 * (L::RW + 1) + 3) & ~3u);
 }
 template <class L>
-constexpr uint32_t vs_words() { return S_PIPE * 32 * L::RW + 3 * S_PIPE * 32; }  // row ring + metadata ring
+constexpr uint32_t vs_words() {  // row ring + metadata ring (+ edge ring and its window rows)
+    return S_PIPE * 32 * L::RW + 3 * S_PIPE * 32 + (edge_smem<L>() ? 2 * S_PIPE * 32 * 3 : 0);
+}
 
 template <int KIND, bool PACKED, class L>
 __global__ void __launch_bounds__(BT, BT <= 512 ? 512 / BT : 1) batch_kernel(BParams P) {
@@ -1703,7 +1832,8 @@ void launch_b(const BParams& P, int sms, cudaStream_t s) {
     // the certificates' source hub values (sh) only when the call uses them: shared memory not
     // allocated stays L1
     const size_t base = (size_t)BW * (xs_words<L>() + vs_words<L>()) * sizeof(uint32_t);
-    const size_t smax = base + (size_t)L::Q * 2 * 64 * sizeof(uint32_t);
+    constexpr bool HUBS = L::QPW == 1 && L::RW > 1;  // u32 lanes: the only ones given hub certificates
+    const size_t smax = base + (HUBS ? (size_t)L::Q * 2 * 64 * sizeof(uint32_t) : 0u);
     const size_t smem = P.HB ? smax : base;
     static int bps = 0;
     if (!bps) {
