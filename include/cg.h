@@ -234,15 +234,30 @@ cg_status cg_graph_status(cg_graph g, void* stream);
 
 /*
  * End-to-end variant with HOST buffers: src (host, n_src ids) and out (host, n_src*n words).
- * Copies sources host->device, runs the queries in device batches of `batch` (<= 0: auto)
- * and streams each batch's values device->host while the next batch computes (two internal
- * streams ordered after `stream`).  Synchronises `stream` before returning.
+ * Copies sources host->device, runs the queries in device batches of `batch` (<= 0: about 512 MiB
+ * of result rows, rounded down to whole passes of the batched engine — 32 queries, 16 for u32 lanes)
+ * and streams each batch's values device->host on the graph's copy stream while the next batch
+ * computes (two device result slots, kept by the graph between calls).  Synchronises `stream`
+ * before returning; out is complete and the call's device errors are returned.
  */
 cg_status cg_query_host(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode, void* out,
                         int32_t batch, void* stream);
 /* The same with an output format (cg_out_format): out (host) holds n_src rows in that format. */
 cg_status cg_query_host_fmt(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode,
                             cg_out_format fmt, void* out, int32_t batch, void* stream);
+
+/*
+ * Asynchronous cg_query_host_fmt: enqueues the source copy, the queries and the result copies and
+ * returns without synchronising.  `stream` is made to wait for the call's last device->host copy,
+ * so out is complete once `stream` is (cudaStreamSynchronize, or cg_graph_status which also
+ * returns the call's device errors; otherwise they are returned by the next call on the graph).
+ * out must be pinned host memory for the copies to overlap and stay valid until `stream`
+ * completes; src (any host memory) is staged before the call returns.  The result copies of one call overlap the computation of the next call on
+ * the graph (a multi-kind step drains kind k's rows while kind k+1 computes).  Host-checkable
+ * errors return at once, as for the synchronous call.
+ */
+cg_status cg_query_host_async(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode,
+                              cg_out_format fmt, void* out, int32_t batch, void* stream);
 
 /*
  * Device twin of the seeded R-MAT input generator (gen/rmat.c defines it): edges

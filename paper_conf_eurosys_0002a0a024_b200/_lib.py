@@ -94,6 +94,8 @@ _SIGS = {
     "cg_query_host": (ctypes.c_int, [_P, ctypes.c_int, _P, ctypes.c_int32, ctypes.c_int, _P, ctypes.c_int32, _P]),
     "cg_query_host_fmt": (ctypes.c_int, [_P, ctypes.c_int, _P, ctypes.c_int32, ctypes.c_int, ctypes.c_int, _P,
                                          ctypes.c_int32, _P]),
+    "cg_query_host_async": (ctypes.c_int, [_P, ctypes.c_int, _P, ctypes.c_int32, ctypes.c_int, ctypes.c_int, _P,
+                                         ctypes.c_int32, _P]),
     "cg_rmat_generate": (ctypes.c_int, [ctypes.c_uint64, ctypes.c_uint32, ctypes.c_uint32, ctypes.c_uint32,
                                         ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int32, ctypes.c_uint64,
                                         ctypes.c_uint64, _P, _P, _P, _P]),

@@ -380,63 +380,98 @@ cg_status cg_graph_status(cg_graph g, void* stream) {
     });
 }
 
+// The host path (cg_query_host*): sources host -> device, the queries in device batches of `batch`,
+// each batch's rows device -> host on the graph's copy stream while the next batch computes.  The
+// result slots, the device sources and the copy stream persist in the graph (HostPath), so an
+// asynchronous call returns with its copies still in flight and the NEXT call (another kind, say)
+// computes while they drain; slot reuse is ordered by events (done / drained), across calls too.
+// At the end the call's stream waits for its last copy: synchronising `stream` completes `out`.
+static void query_host(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode, cg_out_format fmt,
+                       void* out, int32_t batch, void* stream, bool sync) {
+    prepare_query(g, kind, n_src, mode, out, src);
+    check_format(kind, fmt);
+    if (n_src == 0) return;
+    Graph& G = g->G;
+    if (kind == CG_WCC) src = nullptr;
+    if (src) check_sources_host(G, src, n_src);
+    CGB_CUDA(cudaSetDevice(G.device));
+    cudaStream_t s = S(stream);
+    order_begin(G, s);
+    if (kind == CG_WCC) ensure_wcc_graphs(G, mode == CG_MODE_2PHASE, s);
+    const size_t row = row_bytes_of(G, fmt);
+    if (batch <= 0) {  // ~512 MiB of results per batch, rounded down to whole engine passes, at least 1 query
+        size_t b = ((size_t)512 << 20) / (row ? row : 1);
+        const size_t pw = (size_t)pass_width(G, kind);
+        if (b >= pw) b -= b % pw;
+        batch = (int32_t)(b < 1 ? 1 : (b > (size_t)n_src ? (size_t)n_src : b));
+    }
+    if (batch > n_src) batch = n_src;
+    HostPath& h = G.hp;
+    if (!h.cp) {
+        CGB_CUDA(cudaStreamCreateWithFlags(&h.cp, cudaStreamNonBlocking));
+        for (int i = 0; i < 2; ++i) {
+            CGB_CUDA(cudaEventCreateWithFlags(&h.done[i], cudaEventDisableTiming));
+            CGB_CUDA(cudaEventCreateWithFlags(&h.drained[i], cudaEventDisableTiming));
+        }
+        CGB_CUDA(cudaEventCreateWithFlags(&h.src_copied, cudaEventDisableTiming));
+    }
+    const size_t need = (size_t)batch * row;
+    for (int k = 0; k < 2; ++k) {
+        if (h.slot[k].n >= need) continue;
+        if (h.pending[k]) CGB_CUDA(cudaEventSynchronize(h.drained[k]));  // a copy may still read the old slot
+        h.slot[k].alloc(need, s);
+        h.pending[k] = false;
+    }
+    if (src) {  // host -> pinned staging -> device: an asynchronous copy whatever memory src is in
+        if (h.src_pending) CGB_CUDA(cudaEventSynchronize(h.src_copied));  // the staging's previous copy is done
+        h.src_pending = false;
+        if (h.hsrc_n < (size_t)n_src) {
+            if (h.hsrc) CGB_CUDA(cudaFreeHost(h.hsrc));
+            h.hsrc = nullptr;
+            h.hsrc_n = 0;
+            CGB_CUDA(cudaMallocHost(&h.hsrc, 4ull * n_src));
+            h.hsrc_n = (size_t)n_src;
+        }
+        memcpy(h.hsrc, src, 4ull * n_src);
+        if (h.dsrc.n < (size_t)n_src) h.dsrc.alloc((size_t)n_src, s);  // stream-ordered after its last reader
+        CGB_CUDA(cudaMemcpyAsync(h.dsrc.get(), h.hsrc, 4ull * n_src, cudaMemcpyHostToDevice, s));
+        CGB_CUDA(cudaEventRecord(h.src_copied, s));
+        h.src_pending = true;
+    }
+    const bool two = mode == CG_MODE_2PHASE;
+    int last = 0;
+    for (int32_t q0 = 0; q0 < n_src; q0 += batch) {
+        const int32_t nq = (n_src - q0) < batch ? (n_src - q0) : batch;
+        const int k = h.next;
+        h.next ^= 1;
+        if (h.pending[k]) CGB_CUDA(cudaStreamWaitEvent(s, h.drained[k], 0));  // slot k's previous rows copied out
+        QueryCall c = make_call(G, kind, two, src ? h.dsrc.get() + q0 : nullptr, nq, h.slot[k].get(), nullptr, false,
+                                fmt);
+        run_queries(G, c, s, nullptr);
+        CGB_CUDA(cudaEventRecord(h.done[k], s));
+        CGB_CUDA(cudaStreamWaitEvent(h.cp, h.done[k], 0));
+        CGB_CUDA(cudaMemcpyAsync((uint8_t*)out + (size_t)q0 * row, h.slot[k].get(), (size_t)nq * row,
+                                 cudaMemcpyDeviceToHost, h.cp));
+        CGB_CUDA(cudaEventRecord(h.drained[k], h.cp));
+        h.pending[k] = true;
+        last = k;
+    }
+    CGB_CUDA(cudaStreamWaitEvent(s, h.drained[last], 0));  // `stream` completes only after every copy of the call
+    order_end(G, s);
+    if (sync) {
+        CGB_CUDA(cudaStreamSynchronize(s));
+        take_sticky(G);
+    }
+}
+
 cg_status cg_query_host_fmt(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode,
                             cg_out_format fmt, void* out, int32_t batch, void* stream) {
-    return guard([&] {
-        prepare_query(g, kind, n_src, mode, out, src);
-        check_format(kind, fmt);
-        if (n_src == 0) return;
-        Graph& G = g->G;
-        if (kind == CG_WCC) src = nullptr;
-        if (src) check_sources_host(G, src, n_src);
-        CGB_CUDA(cudaSetDevice(G.device));
-        cudaStream_t s = S(stream);
-        order_begin(G, s);
-        if (kind == CG_WCC) ensure_wcc_graphs(G, mode == CG_MODE_2PHASE, s);
-        const size_t row = row_bytes_of(G, fmt);
-        if (batch <= 0) {  // ~256 MiB of results per batch, at least 1 query
-            size_t b = ((size_t)256 << 20) / (row ? row : 1);
-            batch = (int32_t)(b < 1 ? 1 : (b > (size_t)n_src ? (size_t)n_src : b));
-        }
-        if (batch > n_src) batch = n_src;
-        DevBuf<uint32_t> dsrc((size_t)n_src, s);
-        if (src) CGB_CUDA(cudaMemcpyAsync(dsrc.get(), src, 4ull * n_src, cudaMemcpyHostToDevice, s));
-        // two result slots: batch b computes on `s` into slot b%2 while batch b-1 drains on `cp`
-        DevBuf<uint8_t> slot[2];
-        slot[0].alloc((size_t)batch * row, s);
-        if (n_src > batch) slot[1].alloc((size_t)batch * row, s);
-        cudaStream_t cp;
-        CGB_CUDA(cudaStreamCreateWithFlags(&cp, cudaStreamNonBlocking));
-        cudaEvent_t done[2], drained[2];
-        for (int i = 0; i < 2; ++i) {
-            CGB_CUDA(cudaEventCreateWithFlags(&done[i], cudaEventDisableTiming));
-            CGB_CUDA(cudaEventCreateWithFlags(&drained[i], cudaEventDisableTiming));
-        }
-        const bool two = mode == CG_MODE_2PHASE;
-        int b = 0;
-        for (int32_t q0 = 0; q0 < n_src; q0 += batch, ++b) {
-            const int32_t nq = (n_src - q0) < batch ? (n_src - q0) : batch;
-            const int k = b & 1;
-            if (b >= 2) CGB_CUDA(cudaStreamWaitEvent(s, drained[k], 0));
-            QueryCall c = make_call(G, kind, two, src ? dsrc.get() + q0 : nullptr, nq, slot[k].get(), nullptr, false,
-                                    fmt);
-            run_queries(G, c, s, nullptr);
-            CGB_CUDA(cudaEventRecord(done[k], s));
-            CGB_CUDA(cudaStreamWaitEvent(cp, done[k], 0));
-            CGB_CUDA(cudaMemcpyAsync((uint8_t*)out + (size_t)q0 * row, slot[k].get(), (size_t)nq * row,
-                                     cudaMemcpyDeviceToHost, cp));
-            CGB_CUDA(cudaEventRecord(drained[k], cp));
-        }
-        CGB_CUDA(cudaStreamSynchronize(cp));
-        CGB_CUDA(cudaStreamSynchronize(s));
-        order_end(G, s);
-        for (int i = 0; i < 2; ++i) {
-            cudaEventDestroy(done[i]);
-            cudaEventDestroy(drained[i]);
-        }
-        cudaStreamDestroy(cp);
-        take_sticky(G);
-    });
+    return guard([&] { query_host(g, kind, src, n_src, mode, fmt, out, batch, stream, true); });
+}
+
+cg_status cg_query_host_async(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode,
+                              cg_out_format fmt, void* out, int32_t batch, void* stream) {
+    return guard([&] { query_host(g, kind, src, n_src, mode, fmt, out, batch, stream, false); });
 }
 
 cg_status cg_query_host(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode, void* out,

@@ -2064,6 +2064,12 @@ void run_batched_lw(Graph& G, const QueryCall& c, int lw, cudaStream_t s, std::v
 
 }  // namespace
 
+int pass_width(const Graph& G, int kind) {  // queries one batched-engine pass evaluates together
+    if (!batch_width()) return 1;
+    const int lw = lane_width(G, kind);
+    return lw == 2 ? 1 : lw == 32 ? 16 : 32;
+}
+
 int batch_width() {
     const char* e = getenv("CG_BATCH");
     return (e && atoi(e) == 0) ? 0 : 16;  // CG_BATCH=0: single-query engine (engine.cu)

@@ -104,6 +104,34 @@ struct BatchSpace {         // engine_batch.cu workspace (one batch of queries p
     }
 };
 
+struct HostPath {  // cg_query_host*: persistent result slots, source buffer and copy stream
+    DevBuf<uint8_t> slot[2];  // two device result slots: batch b computes into b % 2 while b - 1 drains
+    DevBuf<uint32_t> dsrc;    // the call's sources on the device
+    cudaStream_t cp = nullptr;                      // device -> host copies
+    cudaEvent_t done[2] = {nullptr, nullptr};       // slot k computed (on the call's stream)
+    cudaEvent_t drained[2] = {nullptr, nullptr};    // slot k copied out (on cp)
+    bool pending[2] = {false, false};               // drained[k] recorded: slot k may still be read
+    int next = 0;                                   // slot of the next batch (across calls)
+    uint32_t* hsrc = nullptr;                       // pinned staging of the sources (any host src works)
+    size_t hsrc_n = 0;
+    cudaEvent_t src_copied = nullptr;               // the staging buffer's last host -> device copy
+    bool src_pending = false;
+    HostPath() = default;
+    HostPath(const HostPath&) = delete;
+    HostPath& operator=(const HostPath&) = delete;
+    ~HostPath() {
+        if (cp) cudaStreamSynchronize(cp);
+        if (src_pending) cudaEventSynchronize(src_copied);
+        if (hsrc) cudaFreeHost(hsrc);
+        if (src_copied) cudaEventDestroy(src_copied);
+        for (int i = 0; i < 2; ++i) {
+            if (done[i]) cudaEventDestroy(done[i]);
+            if (drained[i]) cudaEventDestroy(drained[i]);
+        }
+        if (cp) cudaStreamDestroy(cp);
+    }
+};
+
 struct Graph {
     int device = 0;
     uint32_t n = 0, m = 0, w_max = 0;
@@ -118,6 +146,7 @@ struct Graph {
     bool gsym_built = false;
     Workspace ws;
     BatchSpace bs;
+    HostPath hp;
     // sticky error word of asynchronous calls (ERR_* bits of the engines), in host-mapped pinned
     // memory: kernels write it through sticky_d, the next API call / cg_graph_status reads sticky_h
     uint32_t* sticky_h = nullptr;
@@ -175,6 +204,7 @@ struct QueryCall {
 void run_queries(Graph& G, const QueryCall& c, cudaStream_t s, std::vector<cg_stats>* stats);
 
 // engine_batch.cu
+int pass_width(const Graph& G, int kind);  // queries per batched-engine pass for `kind` (1: single-query engine)
 int batch_width();  // B of the batched engine (CG_BATCH env: 8 / 16 / 32; anything else disables it)
 void run_queries_batched(Graph& G, const QueryCall& c, int B, cudaStream_t s, std::vector<cg_stats>* stats);
 

@@ -242,9 +242,10 @@ class Graph:
         return (res, *extra) if extra else res
 
     def query_host(self, kind, sources, mode: str = "2phase", out: torch.Tensor | None = None,
-                   batch: int = 0, fmt: str = "u32") -> torch.Tensor:
+                   batch: int = 0, fmt: str = "u32", sync: bool = True) -> torch.Tensor:
         """cg_query_host_fmt: host sources in, host (pinned) values out in `fmt`, copies overlapped
-        with compute."""
+        with compute.  sync=False: cg_query_host_async — out (pinned) is complete once the current
+        stream is; keep it alive until then (the sources are staged by the call)."""
         k = kind_id(kind)
         src = sources if isinstance(sources, torch.Tensor) else torch.as_tensor(sources)
         src = src.to(torch.int64).to(torch.uint32).contiguous().cpu()
@@ -253,8 +254,9 @@ class Graph:
             cols, dt = self.row_shape(fmt)
             out = torch.empty((ns, cols), dtype=dt, pin_memory=True)
         with torch.cuda.device(self.device):
-            _lib.call("cg_query_host_fmt", self._h, k, _ptr(src), ns, MODES[mode], FORMATS[fmt], _ptr(out),
-                      int(batch), _stream(self.device))
+            _lib.call("cg_query_host_fmt" if sync else "cg_query_host_async", self._h, k, _ptr(src), ns, MODES[mode],
+                      FORMATS[fmt], _ptr(out), int(batch), _stream(self.device))
+
         return out.view(torch.float32) if (k == KINDS["viterbi"] and fmt == "u32") else out
 
     def status(self) -> None:

@@ -225,3 +225,39 @@ def test_split_core_graph_layout():
         for i, s in enumerate(sources):
             assert_values_equal(out[i], oracle.query(kind, og, int(s)), kind, f"split {kind} s={s}")
     g.close()
+
+
+def test_query_host_async_calls_overlap_and_complete():
+    """cg_query_host_async: six calls of different kinds (and formats) back to back on one graph,
+    each in several device batches so the two result slots are reused within and across calls,
+    one stream synchronisation at the end — every row equals the oracle; a synchronous call and a
+    sticky-error check follow on the same graph."""
+    n, src, dst, w = _rmat(14, 16, 91)
+    g, og = both(n, src, dst, w)
+    sources = gen.sample_sources(n, src, dst, 9, seed=13)
+    fmts = {"sssp": "u16", "sswp": "u32", "ssnp": "u16", "viterbi": "u32", "bfs": "u16", "reach": "bits"}
+    for kind in KINDS:
+        g.build(kind, K=12)
+    outs = {}
+    for i, kind in enumerate(KINDS):
+        cols, dt = g.row_shape(fmts[kind])
+        outs[kind] = torch.empty((len(sources), cols), dtype=dt, pin_memory=True)
+        g.query_host(kind, torch.from_numpy(sources.astype(np.int64)), mode="2phase" if i % 2 == 0 else "full",
+                     out=outs[kind], batch=2 + i % 3, fmt=fmts[kind], sync=False)
+    torch.cuda.current_stream().synchronize()
+    g.status()
+    for kind in KINDS:
+        got = outs[kind]
+        for i, s in enumerate(sources):
+            exp = oracle.query(kind, og, int(s))
+            if fmts[kind] == "u16":
+                assert np.array_equal(got[i].view(torch.int16).numpy().view(np.uint16), _u16_of(exp)), (kind, s)
+            elif fmts[kind] == "bits":
+                assert np.array_equal(got[i].view(torch.int32).numpy().view(np.uint32), _bits_of(exp)), (kind, s)
+            else:
+                assert_values_equal(got[i].view(torch.int32).numpy().view(np.uint32), exp, kind, f"{kind}/async")
+    sync = g.query_host("sssp", torch.from_numpy(sources.astype(np.int64)), mode="2phase", batch=4)
+    for i, s in enumerate(sources):
+        assert_values_equal(sync[i].view(torch.int32).numpy().view(np.uint32), oracle.query("sssp", og, int(s)),
+                            "sssp", "sync after async")
+    g.close()
