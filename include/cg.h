@@ -248,13 +248,13 @@ cg_status cg_query_host_fmt(cg_graph g, cg_kind kind, const uint32_t* src, int32
 
 /*
  * Asynchronous cg_query_host_fmt: enqueues the source copy, the queries and the result copies and
- * returns without synchronising.  `stream` is made to wait for the call's last device->host copy,
- * so out is complete once `stream` is (cudaStreamSynchronize, or cg_graph_status which also
- * returns the call's device errors; otherwise they are returned by the next call on the graph).
- * out must be pinned host memory for the copies to overlap and stay valid until `stream`
- * completes; src (any host memory) is staged before the call returns.  The result copies of one call overlap the computation of the next call on
- * the graph (a multi-kind step drains kind k's rows while kind k+1 computes).  Host-checkable
- * errors return at once, as for the synchronous call.
+ * returns without synchronising.  The result copies run on the graph's own copy stream, so they
+ * overlap the computation of the next call on the graph (a multi-kind step drains kind k's rows
+ * while kind k+1 computes).  out is complete once cg_graph_status(g, stream) returns (it waits for
+ * `stream` and the graph's copy stream, and returns the device errors of the calls), or once a
+ * later synchronous cg_query_host* call on the graph returns; synchronising `stream` alone is not
+ * enough.  out must be pinned host memory for the copies to overlap and stay valid until then;
+ * src (any host memory) is staged before the call returns.  Host-checkable errors return at once.
  */
 cg_status cg_query_host_async(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_src, cg_mode mode,
                               cg_out_format fmt, void* out, int32_t batch, void* stream);

@@ -376,6 +376,7 @@ cg_status cg_graph_status(cg_graph g, void* stream) {
         CGB_CHECK(g != nullptr, CG_EINVAL, "null graph");
         CGB_CUDA(cudaSetDevice(g->G.device));
         CGB_CUDA(cudaStreamSynchronize(S(stream)));
+        if (g->G.hp.cp) CGB_CUDA(cudaStreamSynchronize(g->G.hp.cp));  // asynchronous host calls' result copies
         take_sticky(g->G);
     });
 }
@@ -413,7 +414,7 @@ static void query_host(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_
             CGB_CUDA(cudaEventCreateWithFlags(&h.done[i], cudaEventDisableTiming));
             CGB_CUDA(cudaEventCreateWithFlags(&h.drained[i], cudaEventDisableTiming));
         }
-        CGB_CUDA(cudaEventCreateWithFlags(&h.src_copied, cudaEventDisableTiming));
+        for (int i = 0; i < 2; ++i) CGB_CUDA(cudaEventCreateWithFlags(&h.src_copied[i], cudaEventDisableTiming));
     }
     const size_t need = (size_t)batch * row;
     for (int k = 0; k < 2; ++k) {
@@ -422,21 +423,23 @@ static void query_host(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_
         h.slot[k].alloc(need, s);
         h.pending[k] = false;
     }
-    if (src) {  // host -> pinned staging -> device: an asynchronous copy whatever memory src is in
-        if (h.src_pending) CGB_CUDA(cudaEventSynchronize(h.src_copied));  // the staging's previous copy is done
-        h.src_pending = false;
-        if (h.hsrc_n < (size_t)n_src) {
-            if (h.hsrc) CGB_CUDA(cudaFreeHost(h.hsrc));
-            h.hsrc = nullptr;
-            h.hsrc_n = 0;
-            CGB_CUDA(cudaMallocHost(&h.hsrc, 4ull * n_src));
-            h.hsrc_n = (size_t)n_src;
+    if (src) {  // host -> pinned staging (two buffers, alternating) -> device: asynchronous for any src
+        const int k = h.src_next;
+        h.src_next ^= 1;
+        if (h.src_pending[k]) CGB_CUDA(cudaEventSynchronize(h.src_copied[k]));  // that buffer's last copy is done
+        h.src_pending[k] = false;
+        if (h.hsrc_n[k] < (size_t)n_src) {
+            if (h.hsrc[k]) CGB_CUDA(cudaFreeHost(h.hsrc[k]));
+            h.hsrc[k] = nullptr;
+            h.hsrc_n[k] = 0;
+            CGB_CUDA(cudaMallocHost(&h.hsrc[k], 4ull * n_src));
+            h.hsrc_n[k] = (size_t)n_src;
         }
-        memcpy(h.hsrc, src, 4ull * n_src);
+        memcpy(h.hsrc[k], src, 4ull * n_src);
         if (h.dsrc.n < (size_t)n_src) h.dsrc.alloc((size_t)n_src, s);  // stream-ordered after its last reader
-        CGB_CUDA(cudaMemcpyAsync(h.dsrc.get(), h.hsrc, 4ull * n_src, cudaMemcpyHostToDevice, s));
-        CGB_CUDA(cudaEventRecord(h.src_copied, s));
-        h.src_pending = true;
+        CGB_CUDA(cudaMemcpyAsync(h.dsrc.get(), h.hsrc[k], 4ull * n_src, cudaMemcpyHostToDevice, s));
+        CGB_CUDA(cudaEventRecord(h.src_copied[k], s));
+        h.src_pending[k] = true;
     }
     const bool two = mode == CG_MODE_2PHASE;
     int last = 0;
@@ -456,10 +459,11 @@ static void query_host(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_
         h.pending[k] = true;
         last = k;
     }
-    CGB_CUDA(cudaStreamWaitEvent(s, h.drained[last], 0));  // `stream` completes only after every copy of the call
+    (void)last;  // the call's copies complete on h.cp; cg_graph_status / a synchronous call wait for them
     order_end(G, s);
     if (sync) {
         CGB_CUDA(cudaStreamSynchronize(s));
+        CGB_CUDA(cudaStreamSynchronize(h.cp));
         take_sticky(G);
     }
 }

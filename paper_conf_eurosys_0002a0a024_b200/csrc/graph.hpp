@@ -112,18 +112,21 @@ struct HostPath {  // cg_query_host*: persistent result slots, source buffer and
     cudaEvent_t drained[2] = {nullptr, nullptr};    // slot k copied out (on cp)
     bool pending[2] = {false, false};               // drained[k] recorded: slot k may still be read
     int next = 0;                                   // slot of the next batch (across calls)
-    uint32_t* hsrc = nullptr;                       // pinned staging of the sources (any host src works)
-    size_t hsrc_n = 0;
-    cudaEvent_t src_copied = nullptr;               // the staging buffer's last host -> device copy
-    bool src_pending = false;
+    uint32_t* hsrc[2] = {nullptr, nullptr};         // pinned staging of the sources (any host src works)
+    size_t hsrc_n[2] = {0, 0};
+    cudaEvent_t src_copied[2] = {nullptr, nullptr}; // each staging buffer's last host -> device copy
+    bool src_pending[2] = {false, false};
+    int src_next = 0;
     HostPath() = default;
     HostPath(const HostPath&) = delete;
     HostPath& operator=(const HostPath&) = delete;
     ~HostPath() {
         if (cp) cudaStreamSynchronize(cp);
-        if (src_pending) cudaEventSynchronize(src_copied);
-        if (hsrc) cudaFreeHost(hsrc);
-        if (src_copied) cudaEventDestroy(src_copied);
+        for (int i = 0; i < 2; ++i) {
+            if (src_pending[i]) cudaEventSynchronize(src_copied[i]);
+            if (hsrc[i]) cudaFreeHost(hsrc[i]);
+            if (src_copied[i]) cudaEventDestroy(src_copied[i]);
+        }
         for (int i = 0; i < 2; ++i) {
             if (done[i]) cudaEventDestroy(done[i]);
             if (drained[i]) cudaEventDestroy(drained[i]);

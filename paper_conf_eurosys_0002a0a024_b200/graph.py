@@ -244,8 +244,8 @@ class Graph:
     def query_host(self, kind, sources, mode: str = "2phase", out: torch.Tensor | None = None,
                    batch: int = 0, fmt: str = "u32", sync: bool = True) -> torch.Tensor:
         """cg_query_host_fmt: host sources in, host (pinned) values out in `fmt`, copies overlapped
-        with compute.  sync=False: cg_query_host_async — out (pinned) is complete once the current
-        stream is; keep it alive until then (the sources are staged by the call)."""
+        with compute.  sync=False: cg_query_host_async — out (pinned) is complete after
+        `self.status()` (cg_graph_status); keep it alive until then (the sources are staged)."""
         k = kind_id(kind)
         src = sources if isinstance(sources, torch.Tensor) else torch.as_tensor(sources)
         src = src.to(torch.int64).to(torch.uint32).contiguous().cpu()

@@ -230,8 +230,8 @@ def test_split_core_graph_layout():
 def test_query_host_async_calls_overlap_and_complete():
     """cg_query_host_async: six calls of different kinds (and formats) back to back on one graph,
     each in several device batches so the two result slots are reused within and across calls,
-    one stream synchronisation at the end — every row equals the oracle; a synchronous call and a
-    sticky-error check follow on the same graph."""
+    one cg_graph_status at the end — every row equals the oracle; a synchronous call follows on the
+    same graph."""
     n, src, dst, w = _rmat(14, 16, 91)
     g, og = both(n, src, dst, w)
     sources = gen.sample_sources(n, src, dst, 9, seed=13)
@@ -244,8 +244,7 @@ def test_query_host_async_calls_overlap_and_complete():
         outs[kind] = torch.empty((len(sources), cols), dtype=dt, pin_memory=True)
         g.query_host(kind, torch.from_numpy(sources.astype(np.int64)), mode="2phase" if i % 2 == 0 else "full",
                      out=outs[kind], batch=2 + i % 3, fmt=fmts[kind], sync=False)
-    torch.cuda.current_stream().synchronize()
-    g.status()
+    g.status()  # waits for the stream and the graph's copy stream
     for kind in KINDS:
         got = outs[kind]
         for i, s in enumerate(sources):
