@@ -98,6 +98,10 @@ struct BParams {
 //   src_val(), nb_val(w) SourceInitVal and SourceInitVal (+) w, encoded (Alg 3 l.5, l.8)
 //   relax(p, uw, cw, w, act, ...)  Process + EdgeFunction of one word (Alg 3 l.22-27): the lanes
 //       of act whose candidate ext(uw, w) is better than cw; returns the changed lanes
+// RN(1/w) for w = 0..64 (Viterbi's per-edge reciprocal, reading N5): one shared-memory load per edge
+// instead of an IEEE-rounded reciprocal sequence; filled by each CTA at kernel start (exact: __frcp_rn)
+__shared__ float s_rcp[65];
+
 template <int KIND, int QN>
 struct Lanes32 {  // one u32 per query (Table 6 types), QN queries per pass, CGB_G32 words per relax group
     using O = Op<KIND>;
@@ -115,7 +119,7 @@ struct Lanes32 {  // one u32 per query (Table 6 types), QN queries per pass, CGB
     static constexpr bool VIT = KIND == CG_VITERBI;
     using Arg = typename std::conditional<VIT, VitArg, uint32_t>::type;  // per-edge, shared by the row
     __device__ static Arg arg(uint32_t w) {
-        if constexpr (VIT) return vit_arg(w);
+        if constexpr (VIT) return VitArg{w, w <= 64u ? s_rcp[w] : 0.0f};  // RN(1/w) from the CTA's table
         else return w;
     }
     // the pull (phase 1 over CG^R): one query's candidate from u's word, the select of two words
@@ -1627,6 +1631,8 @@ __global__ void __launch_bounds__(BT, BT <= 512 ? 512 / BT : 1) batch_kernel(BPa
     __shared__ uint32_t sm_err;
     __shared__ unsigned long long sm_t[4];  // pass start, phase switch, phase 2 start, values written
     if (threadIdx.x == 0) sm_err = 0u;
+    if (threadIdx.x <= 64) s_rcp[threadIdx.x] = threadIdx.x ? __frcp_rn((float)threadIdx.x) : 0.0f;
+    __syncthreads();
 
     // kernel-level trace marks (tid 0): [cap-1] = {entry, seeds done, loop done, exit} of batch 0
     unsigned long long* kt = (P.trace && tid == 0) ? P.trace + 5ull * (P.trace_cap - 1) : nullptr;

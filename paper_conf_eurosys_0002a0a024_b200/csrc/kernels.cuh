@@ -51,7 +51,7 @@ struct VitArg {
     uint32_t w;
     float r;  // RN(1/w), or 0 (slow path)
 };
-__device__ __forceinline__ VitArg vit_arg(uint32_t w) { return {w, w <= 64u ? __frcp_rn((float)w) : 0.0f}; }
+// (the batched engine builds it as {w, w <= 64 ? RN(1/w) : 0} from a per-CTA table, engine_batch.cu s_rcp)
 __device__ __forceinline__ uint32_t vit_div(uint32_t a, const VitArg& A) {
     const float x = __uint_as_float(a);
     const float b = __uint2float_rn(A.w);  // exact for w <= 64

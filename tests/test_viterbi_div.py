@@ -65,7 +65,11 @@ def test_fast_division_is_correctly_rounded(lib, exp):
 
 def test_fast_path_guard_matches_kernel():
     """The constants the proof above relies on are the ones the kernel uses."""
-    src = open(os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
-                            "paper_conf_eurosys_0002a0a024_b200", "csrc", "kernels.cuh")).read()
-    assert "w <= 64u ? __frcp_rn((float)w)" in src
+    csrc = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
+                        "paper_conf_eurosys_0002a0a024_b200", "csrc")
+    src = open(os.path.join(csrc, "kernels.cuh")).read()
+    eng = open(os.path.join(csrc, "engine_batch.cu")).read()
+    assert "w <= 64u ? s_rcp[w] : 0.0f" in eng                                           # fast path: w <= 64
+    assert "s_rcp[threadIdx.x] = threadIdx.x ? __frcp_rn((float)threadIdx.x) : 0.0f" in eng  # r = RN(1/w)
+    assert "threadIdx.x <= 64" in eng                                                      # table covers 0..64
     assert "x >= 0x1p-64f" in src
