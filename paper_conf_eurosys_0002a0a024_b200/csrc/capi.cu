@@ -442,7 +442,6 @@ static void query_host(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_
         h.src_pending[k] = true;
     }
     const bool two = mode == CG_MODE_2PHASE;
-    int last = 0;
     for (int32_t q0 = 0; q0 < n_src; q0 += batch) {
         const int32_t nq = (n_src - q0) < batch ? (n_src - q0) : batch;
         const int k = h.next;
@@ -457,10 +456,8 @@ static void query_host(cg_graph g, cg_kind kind, const uint32_t* src, int32_t n_
                                  cudaMemcpyDeviceToHost, h.cp));
         CGB_CUDA(cudaEventRecord(h.drained[k], h.cp));
         h.pending[k] = true;
-        last = k;
     }
-    (void)last;  // the call's copies complete on h.cp; cg_graph_status / a synchronous call wait for them
-    order_end(G, s);
+    order_end(G, s);  // the call's copies complete on h.cp: cg_graph_status / a synchronous call wait for them
     if (sync) {
         CGB_CUDA(cudaStreamSynchronize(s));
         CGB_CUDA(cudaStreamSynchronize(h.cp));
