@@ -1552,7 +1552,9 @@ __device__ void transpose_out(const BParams& P, uint32_t* dst, int q0, int nq, u
 // 32 vertices (a tile) per warp: the tile's rows through the padded shared tile (U16), or the
 // 32 x 32 bit matrix of a REACH tile transposed with one ballot per query (BITS).
 template <class L>
-__device__ void transpose_narrow(const BParams& P, int q0, int nq, uint32_t* xs) {
+constexpr uint32_t vs_words();
+template <class L>
+__device__ void transpose_narrow(const BParams& P, int q0, int nq, uint32_t* xs, uint32_t* buf) {
     constexpr int RW = L::RW;
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t gw = blockIdx.x * BW + (threadIdx.x >> 5);
@@ -1575,25 +1577,41 @@ __device__ void transpose_narrow(const BParams& P, int q0, int nq, uint32_t* xs)
       }
     }
     if (P.out_fmt != CG_OUT_U16) return;
+    static_assert(65 * (L::RW + 1) <= vs_words<L>(), "the u16 tile fits the warp's row ring");
     uint16_t* dst = static_cast<uint16_t*>(P.out);
     bool over = false;
-    for (uint32_t tile = gw; tile < T; tile += NW) {
+    // 64 vertices per warp tile, every row written with 4 B stores of vertex PAIRS (128 B per warp
+    // instruction): a pair must start at an even u16 index of the output, so a row whose start
+    // (q0 + q) * n is odd pairs (t0 - 1, t0), (t0 + 1, t0 + 2), ...: the tile's buffer holds the 65
+    // value rows of vertices t0 - 1 .. t0 + 63 (row stride RW + 1 words), and one more tile than
+    // n / 64 covers the last vertex of the odd rows.  Unpaired ends use a 2 B store.
+    constexpr uint32_t RP = RW + 1;
+    const uint32_t T2 = P.n / 64 + 1;
+    auto val16 = [&](uint32_t r, int q) -> uint32_t {
+        const uint32_t x = L::decode(buf[r * RP + q / L::QPW], q % L::QPW);
+        over |= x >= 0xffffu && x != 0xffffffffu;
+        return x >= 0xffffu ? 0xffffu : x;
+    };
+    for (uint32_t tile = gw; tile < T2; tile += NW) {
+        const uint32_t t0 = tile * 64;
         __syncwarp();
 #pragma unroll
-        for (int r = 0; r < RW; ++r) {
-            const uint32_t f = r * 32 + lane;
-            const uint32_t v = tile * 32 + f / RW;
-            xs[(f / RW) * (RW + 1) + f % RW] = v < P.n ? __ldcg(P.V + (size_t)v * RW + f % RW) : 0u;
+        for (uint32_t f = lane; f < 65u * RW; f += 32) {  // buffer row r = vertex t0 - 1 + r
+            const uint32_t r = f / RW, wd = f % RW, v = t0 - 1u + r;  // (t0 = 0, r = 0: v wraps past n)
+            buf[r * RP + wd] = v < P.n ? __ldcg(P.V + (size_t)v * RW + wd) : 0u;
         }
         __syncwarp();
-        const uint32_t v = tile * 32 + lane;
-        if (v < P.n)
-            for (int q = 0; q < nq; ++q) {
-                const uint32_t x = L::decode(xs[lane * (RW + 1) + q / L::QPW], q % L::QPW);
-                over |= x >= 0xffffu && x != 0xffffffffu;
-                __stcs(reinterpret_cast<unsigned short*>(dst + (size_t)(q0 + q) * P.n + v),
-                       (unsigned short)(x >= 0xffffu ? 0xffffu : x));
-            }
+        for (int q = 0; q < nq; ++q) {
+            const uint64_t base = (uint64_t)(q0 + q) * P.n;
+            const uint32_t par = (uint32_t)(base & 1u);
+            const uint32_t va = t0 + 2 * lane - par;  // the lane's pair: vertices va, va + 1
+            const uint32_t ra = 2 * lane + 1 - par;   // their buffer rows ra, ra + 1
+            const bool oka = va < P.n, okb = va + 1u < P.n;  // (va = -1 wraps past n)
+            const uint32_t lo = val16(ra, q), hi = val16(ra + 1, q);
+            if (oka && okb) __stcs(reinterpret_cast<unsigned int*>(dst + base + va), lo | (hi << 16));
+            else if (oka) __stcs(reinterpret_cast<unsigned short*>(dst + base + va), (unsigned short)lo);
+            else if (okb) __stcs(reinterpret_cast<unsigned short*>(dst + base + (uint32_t)(va + 1u)), (unsigned short)hi);
+        }
     }
     if (over) atomicOr(P.err, ERR_NARROW);
 }
@@ -1798,7 +1816,7 @@ __global__ void __launch_bounds__(BT, BT <= 512 ? 512 / BT : 1) batch_kernel(BPa
             transpose_out<L>(P, static_cast<uint32_t*>(P.out), q0, nq, xs, vs);
         } else {
             if (P.out_fmt == CG_OUT_U32) transpose_out<L>(P, static_cast<uint32_t*>(P.out), q0, nq, xs, vs);
-            else transpose_narrow<L>(P, q0, nq, xs);
+            else transpose_narrow<L>(P, q0, nq, xs, vs);
         }
         if (P.stats) {  // reached / precise per query (the thread's query q is fixed)
             grid_sync(P.ctrl, epoch);  // every CTA's values written: the phase-2 end time

@@ -260,3 +260,26 @@ def test_query_host_async_calls_overlap_and_complete():
         assert_values_equal(sync[i].view(torch.int32).numpy().view(np.uint32), oracle.query("sssp", og, int(s)),
                             "sssp", "sync after async")
     g.close()
+
+
+@pytest.mark.parametrize("n", [4099, 4160, 4161, 63, 1])
+def test_u16_rows_any_alignment(n):
+    """CG_OUT_U16 rows start at u16 index q * n: for odd n every other row starts at an odd index, and
+    the transpose writes vertex pairs with 4 B stores, so rows of both parities, tiles ending exactly
+    at n (n = 64 k, 64 k + 1), tiny graphs and ragged batches (33, 45 sources: two passes, the last
+    partial) must all hold the oracle's values."""
+    rng = np.random.default_rng(n)
+    m = 8 * n
+    src = rng.integers(0, n, m).astype(np.uint32)
+    dst = rng.integers(0, n, m).astype(np.uint32)
+    w = rng.integers(1, 24, m).astype(np.uint32)
+    g, og = both(n, src, dst, w)
+    for ns in (33, 45):
+        sources = rng.integers(0, n, ns).astype(np.uint32)
+        for kind in ("sssp", "bfs", "reach"):
+            g.build(kind, K=min(8, n))
+            for mode in ("2phase", "full"):
+                got = u16np(g.query(kind, to_dev(sources), mode=mode, fmt="u16"))
+                for i, s in enumerate(sources):
+                    assert np.array_equal(got[i], _u16_of(oracle.query(kind, og, int(s)))), (n, ns, kind, mode, i)
+    g.close()

@@ -19,6 +19,7 @@ def main():
     p.add_argument("--mode", default="2phase")
     p.add_argument("--batch", type=int, default=32)
     p.add_argument("--repeat", type=int, default=1)
+    p.add_argument("--fmt", default="u32", help="output rows: u32 / u16 / bits (cg_out_format)")
     a = p.parse_args()
     import numpy as np
     import torch
@@ -34,14 +35,15 @@ def main():
     deg = (ptr[1:] - ptr[:-1]).cpu().numpy()
     rng = np.random.default_rng(1000)
     srcs = torch.from_numpy(rng.choice(np.nonzero(deg > 0)[0], size=a.batch).astype(np.int64)).to(torch.uint32).cuda()
-    out = torch.empty((a.batch, cfg.n), dtype=torch.uint32, device="cuda:0")
-    g.query(a.kind, srcs, mode=a.mode, out=out)  # warm
+    cols, dt = g.row_shape(a.fmt)
+    out = torch.empty((a.batch, cols), dtype=dt, device="cuda:0")
+    g.query(a.kind, srcs, mode=a.mode, out=out, fmt=a.fmt)  # warm
     torch.cuda.synchronize()
     for _ in range(a.repeat):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         torch.cuda.nvtx.range_push("prof")
         e0.record()
-        g.query(a.kind, srcs, mode=a.mode, out=out)
+        g.query(a.kind, srcs, mode=a.mode, out=out, fmt=a.fmt)
         e1.record()
         torch.cuda.nvtx.range_pop()
         torch.cuda.synchronize()
