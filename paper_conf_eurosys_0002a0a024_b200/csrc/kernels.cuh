@@ -67,15 +67,19 @@ __device__ __forceinline__ uint32_t vit_div(uint32_t a, const VitArg& A) {
 template <int N>
 __device__ __forceinline__ void vit_div4(const uint32_t (&a)[N], const VitArg& A, uint32_t (&out)[N]) {
     const float b = __uint2float_rn(A.w);
-    bool slow = A.r == 0.0f;
+    // a lane leaves the fast path iff 0 < x < 2^-64 (0 / w = 0 on the fast path too); values are
+    // non-negative binary32, whose bit patterns order like the values and 2^-64 is 0x1F800000, so
+    // that is (bits - 1) < 0x1F7FFFFF unsigned: one min per lane instead of two compares
+    uint32_t lo = 0xffffffffu;
 #pragma unroll
     for (int i = 0; i < N; ++i) {
         const float x = __uint_as_float(a[i]);
         const float q = __fmul_rn(x, A.r);
         const float e = __fmaf_rn(-q, b, x);
         out[i] = __float_as_uint(__fmaf_rn(e, A.r, q));
-        slow |= !(x >= 0x1p-64f) && a[i] != 0u;  // (0 / w = 0 on the fast path too)
+        lo = min(lo, a[i] - 1u);
     }
+    const bool slow = A.r == 0.0f || lo < 0x1F7FFFFFu;
     if (slow) {
 #pragma unroll
         for (int i = 0; i < N; ++i) out[i] = vit_div(a[i], A);

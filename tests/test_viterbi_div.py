@@ -12,6 +12,7 @@ import os
 import subprocess
 import tempfile
 
+import numpy as np
 import pytest
 
 C_SRC = r"""
@@ -72,4 +73,6 @@ def test_fast_path_guard_matches_kernel():
     assert "w <= 64u ? s_rcp[w] : 0.0f" in eng                                           # fast path: w <= 64
     assert "s_rcp[threadIdx.x] = threadIdx.x ? __frcp_rn((float)threadIdx.x) : 0.0f" in eng  # r = RN(1/w)
     assert "threadIdx.x <= 64" in eng                                                      # table covers 0..64
-    assert "x >= 0x1p-64f" in src
+    assert "x >= 0x1p-64f" in src                                                          # vit_div's guard
+    assert "lo < 0x1F7FFFFFu" in src and "lo = min(lo, a[i] - 1u)" in src                  # vit_div4's guard
+    assert np.float32(2.0 ** -64).view(np.uint32) == 0x1F800000                            # = x >= 2^-64
